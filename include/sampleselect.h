@@ -1,0 +1,166 @@
+/*
+ * sampleselect.h -- C ABI of the B200 SampleSelect hot path.
+ *
+ * Method: Ribizel & Anzt, "Approximate and Exact Selection on GPUs",
+ * IPDPS-W 2019 (/root/reference/PAPER.md, cited as L<line>).
+ *
+ * Problem (§II): for an input sequence x_0..x_{n-1}, return the element
+ * at position k (0-based) of the sorted sequence; if a value occurs several
+ * times it carries the smallest rank.  Floating-point values are ordered by
+ * IEEE-754 totalOrder (-NaN < -inf < ... < -0 < +0 < ... < +inf < +NaN;
+ * DESIGN.md reading R3), integers numerically, so the answer is unique
+ * bit-for-bit.  The input is never modified (L237-245).
+ *
+ * Everything below runs in hand-written sm_100a kernels; there is no CPU
+ * fallback.  If no CUDA device is usable every call returns SS_ERR_CUDA.
+ *
+ * Conventions shared by all calls
+ *   - d_* pointers are DEVICE pointers on the context's device; h_* pointers
+ *     are HOST pointers (pageable or pinned).  Device inputs must be
+ *     naturally aligned for their dtype (4 or 8 bytes); any further alignment
+ *     is handled (kernels peel unaligned heads).  Inputs are read-only.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default
+ *     stream).  Calls that return a host result synchronise that stream
+ *     before returning; *_async calls only enqueue work.
+ *   - The context owns all workspace (oracle bytes, survivor buffers, level
+ *     state); it grows lazily and is freed by ss_destroy.  Outputs are
+ *     written only on SS_OK; on error they are untouched and ss_last_error()
+ *     describes the failure.  No C++ exception or abort crosses this ABI.
+ *   - One context per host thread and stream; contexts are independent.
+ */
+#ifndef SAMPLESELECT_H
+#define SAMPLESELECT_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define SS_ABI_VERSION 1
+#define SS_MAX_LEVELS 32
+
+typedef enum { SS_FLOAT32 = 0, SS_FLOAT64 = 1, SS_INT32 = 2, SS_INT64 = 3 } ss_dtype;
+
+typedef enum {
+    SS_OK = 0,
+    SS_ERR_INVALID_ARGUMENT = 1, /* NULL pointer, n < 1, k not in [0,n), bad dtype/b/config */
+    SS_ERR_CUDA = 2,             /* a CUDA runtime error (no device, launch failure, ...) */
+    SS_ERR_OUT_OF_MEMORY = 3,    /* workspace allocation failed */
+    SS_ERR_INTERNAL = 5          /* recursion-depth guard tripped (should not happen) */
+} ss_status;
+
+typedef struct ss_context ss_context;
+
+/* Tuning knobs (§IV.H).  ss_create fills the defaults. */
+typedef struct {
+    int32_t b_exact;      /* buckets per exact level: power of two in [4, 256]
+                             (oracle bytes cap b at 256, L272-276). default 256 */
+    int32_t sample_size;  /* s: 0 = per-b default clamp(16 b, 4096, 16384) (L557-561);
+                             else a power of two in [b, 16384] */
+    int32_t base_case;    /* B: levels with n <= B finish in one CTA (L97, L579-583);
+                             power of two in [256, 16384]. default 16384 */
+    int32_t ctas_per_sm;  /* count/filter grid = ctas_per_sm * #SMs. default 4 */
+    int32_t profile;      /* 1: record CUDA events around every kernel on the call's
+                             stream and report per-kernel device times in ss_stats */
+    uint64_t seed;        /* sampling seed (reading R7). default 0x5A17 */
+} ss_config;
+
+/* Per-call statistics of the last ss_select / ss_approx_select. */
+typedef struct {
+    int32_t levels;                    /* count passes executed (0 = base case only) */
+    int32_t equality_exit;             /* 1 if the answer came from an equality bucket (§IV.C) */
+    int64_t n_level[SS_MAX_LEVELS];    /* n_l entering level l (n_level[levels] = base-case size) */
+    int32_t bucket[SS_MAX_LEVELS];     /* bucket chosen at level l */
+    double bytes_algorithmic;          /* DESIGN.md §Roofline byte model for this call */
+    int32_t launches;                  /* kernels this call launched */
+    int64_t h2d_bytes;                 /* host->device bytes this call copied (host-input calls) */
+    int64_t d2h_bytes;                 /* device->host bytes this call copied (result block) */
+    float ms_kernel[SS_MAX_LEVELS][3]; /* profile=1: device ms of K1 (sample/tree or base
+                                          case), K2 (count+tail), K5 (filter) per level */
+} ss_stats;
+
+/* ---- context --------------------------------------------------------- */
+/* Create a context bound to CUDA device `device` (>= 0). */
+ss_status ss_create(int device, ss_context** out);
+void      ss_destroy(ss_context* ctx);
+ss_status ss_get_config(const ss_context* ctx, ss_config* out);
+ss_status ss_set_config(ss_context* ctx, const ss_config* cfg);
+ss_status ss_last_stats(const ss_context* ctx, ss_stats* out);
+const char* ss_last_error(const ss_context* ctx);
+const char* ss_status_string(ss_status s);
+int       ss_abi_version(void);
+
+/* ---- exact selection (§II; Fig. 1 L95-127; §IV.B-E) --------------
+ * Writes the element of rank k of d_data[0..n) (4 or 8 bytes, the dtype's
+ * bits) to *h_result.  Device input, host result; synchronises `stream`. */
+ss_status ss_select(ss_context* ctx, ss_dtype dt, const void* d_data, int64_t n, int64_t k,
+                    void* h_result, void* stream);
+
+/* Same, input in HOST memory: the call copies it to device workspace on
+ * `stream` (pinned memory makes that copy asynchronous and fast). */
+ss_status ss_select_host(ss_context* ctx, ss_dtype dt, const void* h_data, int64_t n, int64_t k,
+                         void* h_result, void* stream);
+
+/* ---- approximate selection (§II.C; §V.G) ---------------
+ * One level with b buckets (power of two in [4, 1024]): sample, count, and
+ * return the splitter s_i whose rank r_i is closest to k (ties: smaller i),
+ * with its exact rank *h_rank = #{x < s_i} (reading R11). */
+ss_status ss_approx_select(ss_context* ctx, ss_dtype dt, const void* d_data, int64_t n, int64_t k,
+                           int32_t b, void* h_result, int64_t* h_rank, void* stream);
+ss_status ss_approx_select_host(ss_context* ctx, ss_dtype dt, const void* h_data, int64_t n,
+                                int64_t k, int32_t b, void* h_result, int64_t* h_rank, void* stream);
+
+/* ---- single steps of one level (per-kernel parity tests, sharded driver) --
+ * All are asynchronous on `stream` and touch only the buffers passed in.  Keys
+ * are the order-preserving unsigned images of the values (u32 for 4-byte,
+ * u64 for 8-byte dtypes; reading R3), so tree/splitter buffers hold keys.     */
+
+/* K1a (§IV.B-a; reading R7): draw sample slots [slot_begin,
+ * slot_begin+count) of level `level` uniformly with replacement from
+ * d_data[0..n); writes `count` KEYS to d_sample_keys. */
+ss_status ss_step_sample(ss_context* ctx, ss_dtype dt, const void* d_data, int64_t n, int32_t level,
+                         int64_t slot_begin, int64_t count, void* d_sample_keys, void* stream);
+
+/* K1b (§IV.B-a, §IV.C, Fig. 3): sort s sample keys in one
+ * CTA (bitonic, §IV.D), pick splitters s_i = sorted[floor(i s / b)], apply
+ * the equality fix-up if `fixup` != 0, write the heap-ordered tree
+ * d_tree[b-1], the sorted (fixed) splitters d_splitters[b-1] and the
+ * equality flags d_eq[b] (uint8).  s: power of two <= 16384. */
+ss_status ss_step_tree(ss_context* ctx, ss_dtype dt, const void* d_sample_keys, int32_t s, int32_t b,
+                       int32_t fixup, void* d_tree, void* d_splitters, uint8_t* d_eq, void* stream);
+
+/* K2 (§IV.B-b, Fig. 4, §IV.G): classify d_data[0..n) against the tree (keys),
+ * write per-bucket totals d_totals[b] (uint64, overwritten) and, if
+ * d_oracles != NULL (requires b <= 256), the bucket byte of element i to
+ * d_oracles[i]. */
+ss_status ss_step_count(ss_context* ctx, ss_dtype dt, const void* d_data, int64_t n, const void* d_tree,
+                        int32_t b, uint64_t* d_totals, uint8_t* d_oracles, void* stream);
+
+/* K5 (§IV.B-c): stable compaction of the elements i with
+ * d_oracles[i] == bucket into d_out (values, input order).  Writes the
+ * number of elements copied to *d_count (uint64). */
+ss_status ss_step_filter(ss_context* ctx, ss_dtype dt, const void* d_data, int64_t n,
+                         const uint8_t* d_oracles, int32_t bucket, void* d_out, uint64_t* d_count,
+                         void* stream);
+
+/* ---- sharded (multi-GPU) selection support -------------------
+ * The sharded driver (paper_conf_ipps_ribizela19_b200/sharded.py) runs one
+ * process per GPU, exchanges the sample keys (allgather) and bucket totals
+ * (allreduce) with NCCL through torch.distributed, and calls these steps. */
+
+/* K3/K4 (§IV.G; Fig. 1 lines 11-16; reading R6): given GLOBAL bucket
+ * totals d_totals[b] (uint64) and rank k, find the unique j with
+ * r_j <= k < r_{j+1}; write d_out[0]=j, d_out[1]=k-r_j, d_out[2]=totals[j],
+ * d_out[3]=eq[j] (int64[4]); reads the equality flags d_eq[b]. */
+ss_status ss_step_search(ss_context* ctx, const uint64_t* d_totals, int32_t b, int64_t k,
+                         const uint8_t* d_eq, int64_t* d_out, void* stream);
+
+/* Inverse key map: turn `count` keys into values of dtype dt (in place OK). */
+ss_status ss_step_keys_to_values(ss_context* ctx, ss_dtype dt, const void* d_keys, int64_t count,
+                                 void* d_values, void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* SAMPLESELECT_H */

@@ -1,0 +1,210 @@
+"""B200-native SampleSelect (Ribizel & Anzt, "Approximate and Exact Selection
+on GPUs", IPDPS-W 2019).
+
+Thin Python binding over the C ABI in ``include/sampleselect.h`` (argument
+marshalling only; every step runs in the sm_100a kernels of
+``libsampleselect.so``; there is no CPU fallback).
+
+    import torch, paper_conf_ipps_ribizela19_b200 as ss
+    x = torch.rand(1 << 24, device="cuda")
+    v = ss.select(x, k)                  # element of rank k (§II)
+    v, r = ss.approx_select(x, k, 1024)  # approximate value + exact rank (§II.C)
+
+Inputs: 1-D contiguous torch tensors on a CUDA device (float32/float64/
+int32/int64), or numpy arrays in host memory (copied to the device inside the
+call -- the end-to-end path).  Results are numpy scalars with the exact bits.
+"""
+from __future__ import annotations
+
+import ctypes
+import threading
+
+import numpy as np
+
+from . import _abi
+from ._abi import SSConfig, SSError, SSStats
+
+__all__ = ["Context", "select", "approx_select", "default_context", "SSError"]
+
+_NP_DT = {np.dtype(np.float32): _abi.SS_FLOAT32, np.dtype(np.float64): _abi.SS_FLOAT64,
+          np.dtype(np.int32): _abi.SS_INT32, np.dtype(np.int64): _abi.SS_INT64}
+_NP_OF = {v: k for k, v in _NP_DT.items()}
+
+
+def _torch_dt(t):
+    import torch
+    m = {torch.float32: _abi.SS_FLOAT32, torch.float64: _abi.SS_FLOAT64,
+         torch.int32: _abi.SS_INT32, torch.int64: _abi.SS_INT64}
+    if t.dtype not in m:
+        raise TypeError(f"unsupported dtype {t.dtype}; use float32/float64/int32/int64")
+    return m[t.dtype]
+
+
+def _is_tensor(x) -> bool:
+    try:
+        import torch
+        return isinstance(x, torch.Tensor)
+    except ImportError:  # pragma: no cover
+        return False
+
+
+class Context:
+    """One ss_context: a device, its workspace and its tuning knobs."""
+
+    def __init__(self, device: int = 0, **config):
+        self._lib = _abi.lib()
+        self._h = ctypes.c_void_p()
+        rc = self._lib.ss_create(int(device), ctypes.byref(self._h))
+        if rc:
+            raise SSError(rc, f"ss_create(device={device}) failed (is a CUDA device visible?)")
+        self.device = int(device)
+        if config:
+            self.configure(**config)
+
+    # ---------------------------------------------------------- plumbing --
+    def close(self):
+        if self._h:
+            self._lib.ss_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):  # pragma: no cover
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def _check(self, rc: int):
+        if rc:
+            raise SSError(rc, self._lib.ss_last_error(self._h).decode())
+
+    def _stream(self, stream):
+        if stream is not None:
+            return ctypes.c_void_p(stream if isinstance(stream, int) else stream.cuda_stream)
+        import torch
+        return ctypes.c_void_p(torch.cuda.current_stream(self.device).cuda_stream)
+
+    @property
+    def config(self) -> dict:
+        c = SSConfig()
+        self._check(self._lib.ss_get_config(self._h, ctypes.byref(c)))
+        return {f: getattr(c, f) for f, _ in SSConfig._fields_}
+
+    def configure(self, **kw):
+        c = SSConfig(**{**self.config, **kw})
+        self._check(self._lib.ss_set_config(self._h, ctypes.byref(c)))
+
+    def stats(self) -> dict:
+        s = SSStats()
+        self._check(self._lib.ss_last_stats(self._h, ctypes.byref(s)))
+        L = s.levels
+        return {"levels": L, "equality_exit": bool(s.equality_exit),
+                "n_level": list(s.n_level[:L + 1]), "bucket": list(s.bucket[:L]),
+                "bytes_algorithmic": s.bytes_algorithmic, "launches": s.launches,
+                "h2d_bytes": s.h2d_bytes, "d2h_bytes": s.d2h_bytes,
+                "ms_kernel": [list(s.ms_kernel[l]) for l in range(L + 1)]}
+
+    def _args(self, x):
+        """-> (dtype code, pointer, n, numpy dtype, on_device)"""
+        if _is_tensor(x):
+            if not x.is_cuda:
+                raise ValueError("torch tensor must live on a CUDA device (use numpy for host data)")
+            if x.dim() != 1 or not x.is_contiguous():
+                raise ValueError("input must be a 1-D contiguous tensor")
+            if x.device.index != self.device:
+                raise ValueError(f"tensor on cuda:{x.device.index}, context on cuda:{self.device}")
+            dt = _torch_dt(x)
+            return dt, ctypes.c_void_p(x.data_ptr()), x.numel(), _NP_OF[dt], True
+        a = np.asarray(x)
+        if a.ndim != 1 or not a.flags.c_contiguous:
+            raise ValueError("input must be a 1-D contiguous array")
+        if a.dtype not in _NP_DT:
+            raise TypeError(f"unsupported dtype {a.dtype}")
+        return _NP_DT[a.dtype], ctypes.c_void_p(a.ctypes.data), a.size, a.dtype, False
+
+    # ------------------------------------------------------------- API ----
+    def select(self, x, k: int, stream=None):
+        """Element of rank k (0-based; ties take the smallest rank, §II)."""
+        dt, p, n, npdt, dev = self._args(x)
+        out = np.empty(1, dtype=npdt)
+        fn = self._lib.ss_select if dev else self._lib.ss_select_host
+        self._check(fn(self._h, dt, p, n, int(k), ctypes.c_void_p(out.ctypes.data), self._stream(stream)))
+        return out[0]
+
+    def approx_select(self, x, k: int, b: int = 1024, stream=None):
+        """Approximate element of rank ~k with b buckets and its exact rank
+        #{x < value} (§II.C)."""
+        dt, p, n, npdt, dev = self._args(x)
+        out = np.empty(1, dtype=npdt)
+        rank = ctypes.c_int64(0)
+        fn = self._lib.ss_approx_select if dev else self._lib.ss_approx_select_host
+        self._check(fn(self._h, dt, p, n, int(k), int(b), ctypes.c_void_p(out.ctypes.data),
+                       ctypes.byref(rank), self._stream(stream)))
+        return out[0], int(rank.value)
+
+    # -------------------------------------------- single steps (tensors) --
+    def step_sample(self, x, level: int, slot_begin: int, count: int, out_keys, stream=None):
+        dt, p, n, _, _ = self._args(x)
+        self._check(self._lib.ss_step_sample(self._h, dt, p, n, int(level), int(slot_begin), int(count),
+                                             ctypes.c_void_p(out_keys.data_ptr()), self._stream(stream)))
+
+    def step_tree(self, dt_code: int, sample_keys, b: int, fixup: bool, tree, splitters, eq, stream=None):
+        self._check(self._lib.ss_step_tree(self._h, dt_code, ctypes.c_void_p(sample_keys.data_ptr()),
+                                           sample_keys.numel(), int(b), int(bool(fixup)),
+                                           ctypes.c_void_p(tree.data_ptr()),
+                                           ctypes.c_void_p(splitters.data_ptr()),
+                                           ctypes.c_void_p(eq.data_ptr()), self._stream(stream)))
+
+    def step_count(self, x, tree, b: int, totals, oracles=None, stream=None):
+        dt, p, n, _, _ = self._args(x)
+        self._check(self._lib.ss_step_count(self._h, dt, p, n, ctypes.c_void_p(tree.data_ptr()), int(b),
+                                            ctypes.c_void_p(totals.data_ptr()),
+                                            ctypes.c_void_p(oracles.data_ptr() if oracles is not None else 0),
+                                            self._stream(stream)))
+
+    def step_filter(self, x, oracles, bucket: int, out, count, stream=None):
+        dt, p, n, _, _ = self._args(x)
+        self._check(self._lib.ss_step_filter(self._h, dt, p, n, ctypes.c_void_p(oracles.data_ptr()),
+                                             int(bucket), ctypes.c_void_p(out.data_ptr()),
+                                             ctypes.c_void_p(count.data_ptr()), self._stream(stream)))
+
+    def step_search(self, totals, b: int, k: int, eq, out, stream=None):
+        self._check(self._lib.ss_step_search(self._h, ctypes.c_void_p(totals.data_ptr()), int(b), int(k),
+                                             ctypes.c_void_p(eq.data_ptr() if eq is not None else 0),
+                                             ctypes.c_void_p(out.data_ptr()), self._stream(stream)))
+
+    def step_keys_to_values(self, dt_code: int, keys, values, stream=None):
+        self._check(self._lib.ss_step_keys_to_values(self._h, dt_code, ctypes.c_void_p(keys.data_ptr()),
+                                                     keys.numel(), ctypes.c_void_p(values.data_ptr()),
+                                                     self._stream(stream)))
+
+
+_tls = threading.local()
+
+
+def default_context(device: int | None = None) -> Context:
+    """Thread-local context per device (mirrors north_star's select(data, n, k))."""
+    if device is None:
+        import torch
+        device = torch.cuda.current_device()
+    cache = getattr(_tls, "ctx", None)
+    if cache is None:
+        cache = _tls.ctx = {}
+    if device not in cache:
+        cache[device] = Context(device)
+    return cache[device]
+
+
+def _device_of(x):
+    if _is_tensor(x) and x.is_cuda:
+        return x.device.index
+    return None
+
+
+def select(x, k: int):
+    """Element of rank k of x (exact; bit-identical to sort-and-index)."""
+    return default_context(_device_of(x)).select(x, k)
+
+
+def approx_select(x, k: int, b: int = 1024):
+    """(approximate value, its exact rank) with b buckets, one level."""
+    return default_context(_device_of(x)).approx_select(x, k, b)

@@ -1,0 +1,139 @@
+// common.cuh -- device-side building blocks of the B200 SampleSelect path.
+//
+// Order-preserving keys (reading R3): every value is
+// mapped to an unsigned integer whose numeric order is IEEE totalOrder (floats)
+// or numeric order (ints).  All comparisons in the path (Fig. 4 L335 walk,
+// sample sort, base case) are integer compares on these keys, so -0/+0 and
+// NaNs are ordered bit-exactly; the key successor (+1) is the "s_e + eps" of
+// §IV.C L350-354.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace ss {
+
+typedef unsigned long long u64;
+typedef unsigned int u32;
+
+// ---------------------------------------------------------------- keys ----
+template <typename T> struct Traits;
+template <> struct Traits<float> {
+    typedef u32 Key;
+    static __host__ __device__ __forceinline__ Key to_key(u32 u) {
+        return u ^ ((u32)((int)u >> 31) | 0x80000000u);
+    }
+    static __host__ __device__ __forceinline__ u32 from_key(Key k) {
+        return (k & 0x80000000u) ? (k ^ 0x80000000u) : ~k;
+    }
+};
+template <> struct Traits<double> {
+    typedef u64 Key;
+    static __host__ __device__ __forceinline__ Key to_key(u64 u) {
+        return u ^ ((u64)((long long)u >> 63) | 0x8000000000000000ull);
+    }
+    static __host__ __device__ __forceinline__ u64 from_key(Key k) {
+        return (k & 0x8000000000000000ull) ? (k ^ 0x8000000000000000ull) : ~k;
+    }
+};
+template <> struct Traits<int> {
+    typedef u32 Key;
+    static __host__ __device__ __forceinline__ Key to_key(u32 u) { return u ^ 0x80000000u; }
+    static __host__ __device__ __forceinline__ u32 from_key(Key k) { return k ^ 0x80000000u; }
+};
+template <> struct Traits<long long> {
+    typedef u64 Key;
+    static __host__ __device__ __forceinline__ Key to_key(u64 u) { return u ^ 0x8000000000000000ull; }
+    static __host__ __device__ __forceinline__ u64 from_key(Key k) { return k ^ 0x8000000000000000ull; }
+};
+
+// Raw bits type of T (same width as the key).
+template <typename T> struct Bits { typedef typename Traits<T>::Key type; };
+
+template <typename T>
+__device__ __forceinline__ typename Traits<T>::Key load_key(const T* p) {
+    typedef typename Traits<T>::Key K;
+    K raw = __ldg(reinterpret_cast<const K*>(p));
+    return Traits<T>::to_key(raw);
+}
+
+// --------------------------------------------------------- level state ----
+// Device-resident control block, one per recursion level (§IV.E:
+// control stays on the GPU; the paper used CDP, we pre-enqueue early-exiting
+// kernels).  Zeroed by the init kernel at the start of each call.
+struct LevelCtl {
+    u64 n;          // n_l: elements entering level l
+    u64 k;          // k_l: rank within level l
+    u32 ticket;     // count-kernel CTA completion ticket (last CTA runs the tail)
+    u32 bucket;     // bucket j chosen at level l
+    u32 ncta;       // active CTAs of the count/filter grid
+    u32 pad;
+};
+
+struct SelectResult {
+    u64 bits;                 // answer (raw bits of T)
+    long long rank;           // approximate: exact rank #{x < answer}
+    int done;                 // 1 once bits is valid
+    int levels;               // count passes executed
+    int eq_exit;              // answer from an equality bucket (§IV.C)
+    int incomplete;           // final K1 saw n_l > B: host must enqueue more levels
+    long long n_level[32];
+    int bucket[32];
+    long long split_index;    // approximate: 1-based splitter index returned
+};
+
+// ------------------------------------------------------------ chunking ----
+// Element -> CTA mapping shared by the count (K2) and filter (K5) kernels;
+// the filter must see exactly the count's per-CTA ranges so that the K3
+// offsets apply (§IV.G).  Elements [0, head) are peeled so that the
+// vector body starts 16-byte aligned; the body is nvec 16-byte vectors of
+// V = 16/sizeof(T) elements; [tail_begin, n) is the ragged tail.  CTA g owns
+// body vectors [g*vpc, min((g+1)*vpc, nvec)); CTA 0 also owns the head, the
+// last active CTA the tail.
+struct Chunking {
+    u64 head, nvec, tail_begin, vpc;
+    u32 ncta;
+};
+
+template <typename T>
+__host__ __device__ __forceinline__ Chunking make_chunking(const T* p, u64 n, u32 grid, u32 group_vecs) {
+    const u64 V = 16 / sizeof(T);
+    Chunking c;
+    u64 mis = (u64)((uintptr_t)p & 15u);
+    u64 head = mis ? (16 - mis) / sizeof(T) : 0;
+    if (head > n) head = n;
+    c.head = head;
+    c.nvec = (n - head) / V;
+    c.tail_begin = head + c.nvec * V;
+    // at least 16 groups per CTA so tiny levels use few CTAs
+    u64 min_vpc = (u64)group_vecs * 16;
+    u64 want = (c.nvec + grid - 1) / grid;
+    if (want < min_vpc) want = min_vpc;
+    want = (want + group_vecs - 1) / group_vecs * group_vecs;
+    c.vpc = want;
+    u64 nc = (c.nvec + want - 1) / want;
+    if (nc == 0) nc = 1;
+    if (nc > grid) nc = grid;
+    c.ncta = (u32)nc;
+    return c;
+}
+
+// Oracle byte of element i lives at oracle_base + i, with the base shifted so
+// that the body's bytes start 16-byte aligned.
+__host__ __device__ __forceinline__ u64 oracle_pad(u64 head) { return (16 - (head & 15)) & 15; }
+
+// ------------------------------------------------------------ sampling ----
+// Reading R7: SplitMix64 finaliser (Steele/Lea/Flood 2014), counter based.
+__host__ __device__ __forceinline__ u64 splitmix64(u64 x) {
+    u64 z = x + 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+__host__ __device__ __forceinline__ u64 level_base(u64 seed, int level) {
+    return splitmix64(seed + (u64)level * 0xD1B54A32D192ED03ull);
+}
+__device__ __forceinline__ u64 sample_index(u64 base, u64 slot, u64 n) {
+    return __umul64hi(splitmix64(base + slot), n);
+}
+
+}  // namespace ss

@@ -1,0 +1,734 @@
+// sampleselect.cu -- level driver (Layer 1) and the C ABI (include/sampleselect.h).
+//
+// The driver follows Fig. 1 (L95-127) with the recursion control kept on the
+// device (§IV.E): per call it enqueues an init kernel and, per
+// expected level, K1 (sample/tree or base case) -> K2 (count + fused K3/K4
+// tail) -> K5 (filter), all reading their data-dependent sizes from
+// device-resident LevelCtl blocks and exiting early once the answer is known.
+// A final K1 either finishes the base case or flags "incomplete", in which
+// case (rare: an unlucky sample) more levels are enqueued.  One device->host
+// copy per call returns the answer; there is no per-level host round trip.
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <new>
+#include <string>
+
+#include "kernels.cuh"
+#include "sampleselect.h"
+
+using namespace ss;
+
+struct ss_context {
+    int device = 0;
+    int sms = 0;
+    ss_config cfg{};
+    ss_stats stats{};
+    std::string err;
+    uint8_t* d_oracles = nullptr;
+    size_t cap_oracles = 0;
+    void* d_buf[2] = {nullptr, nullptr};
+    size_t cap_buf[2] = {0, 0};
+    void* d_stage = nullptr;
+    size_t cap_stage = 0;
+    LevelCtl* d_ctl = nullptr;
+    SelectResult* d_res = nullptr;
+    u64* d_totals = nullptr;     // [SS_MAX_LEVELS][MAX_B]
+    u32* d_cta_counts = nullptr; // [MAX_GRID][MAX_B]
+    u64* d_offsets = nullptr;    // [MAX_GRID]
+    u64* d_tree = nullptr;       // [SS_MAX_LEVELS][MAX_B] keys (u32 keys use the same bytes)
+    u64* d_spl = nullptr;
+    uint8_t* d_eq = nullptr;     // [SS_MAX_LEVELS][MAX_B]
+    SelectResult* h_res = nullptr;
+    // record of the last ss_step_count (per-CTA counts feed ss_step_filter)
+    const void* step_ptr = nullptr;
+    u64 step_n = 0;
+    int step_b = 0;
+    int step_dt = -1;
+    u32 step_grid = 0;
+    // profile=1: event pairs around every kernel, slot (level, kernel)
+    cudaEvent_t ev[SS_MAX_LEVELS][3][2] = {};
+    bool ev_used[SS_MAX_LEVELS][3] = {};
+    bool ev_ready = false;
+    int launches = 0;
+    int64_t h2d = 0, d2h = 0;   // bytes copied by the current call
+};
+
+static constexpr u32 MAX_GRID = 4096;
+
+namespace {
+
+struct DevGuard {
+    int prev = -1;
+    explicit DevGuard(int d) {
+        if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+        if (prev != d) cudaSetDevice(d);
+    }
+    ~DevGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
+ss_status fail(ss_context* c, ss_status s, const std::string& msg) {
+    if (c) c->err = msg;
+    return s;
+}
+
+#define CK(call)                                                                              \
+    do {                                                                                      \
+        cudaError_t e_ = (call);                                                              \
+        if (e_ != cudaSuccess) {                                                              \
+            (void)cudaGetLastError();                                                         \
+            return fail(c, e_ == cudaErrorMemoryAllocation ? SS_ERR_OUT_OF_MEMORY : SS_ERR_CUDA, \
+                        std::string(#call) + ": " + cudaGetErrorString(e_));                  \
+        }                                                                                     \
+    } while (0)
+
+#define CKLAUNCH(what) CK(cudaGetLastError())
+
+int log2i(int b) {
+    int h = 0;
+    while ((1 << h) < b) ++h;
+    return h;
+}
+bool pow2(long long x) { return x > 0 && (x & (x - 1)) == 0; }
+
+size_t dt_size(ss_dtype dt) {
+    switch (dt) {
+    case SS_FLOAT32: case SS_INT32: return 4;
+    case SS_FLOAT64: case SS_INT64: return 8;
+    default: return 0;
+    }
+}
+
+int sample_size(const ss_config& cfg, int b) {
+    if (cfg.sample_size > 0) return cfg.sample_size;
+    return std::max(4096, std::min(16 * b, 16384));
+}
+
+ss_status grow(ss_context* c, void** p, size_t* cap, size_t need) {
+    if (*cap >= need && *p) return SS_OK;
+    if (*p) {
+        cudaFree(*p);
+        *p = nullptr;
+        *cap = 0;
+    }
+    size_t alloc = need + need / 16 + 256;
+    CK(cudaMalloc(p, alloc));
+    *cap = alloc;
+    return SS_OK;
+}
+
+// count/filter grid: resident CTAs of the count kernel x #SMs (one wave)
+template <typename T, int H>
+u32 count_grid(ss_context* c) {
+    static int occ[64] = {0};
+    int dev = c->device & 63;
+    if (!occ[dev]) {
+        int o = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, count_kernel<T, H>, K2_THREADS, 0);
+        occ[dev] = o > 0 ? o : 1;
+    }
+    u32 per = (u32)std::max(1, std::min(c->cfg.ctas_per_sm, occ[dev]));
+    return std::min<u32>(per * (u32)c->sms, MAX_GRID);
+}
+
+template <typename T>
+ss_status launch_count(ss_context* c, int H, const T* in, CountArgs& a, cudaStream_t st) {
+#define SS_COUNT_CASE(h)                                                     \
+    case h:                                                                  \
+        a.grid = count_grid<T, h>(c);                                        \
+        count_kernel<T, h><<<a.grid, K2_THREADS, 0, st>>>(in, a);            \
+        break;
+    switch (H) {
+        SS_COUNT_CASE(2) SS_COUNT_CASE(3) SS_COUNT_CASE(4) SS_COUNT_CASE(5) SS_COUNT_CASE(6)
+        SS_COUNT_CASE(7) SS_COUNT_CASE(8) SS_COUNT_CASE(9) SS_COUNT_CASE(10)
+    default: return fail(c, SS_ERR_INVALID_ARGUMENT, "b must be a power of two in [4, 1024]");
+    }
+#undef SS_COUNT_CASE
+    CKLAUNCH("count_kernel");
+    return SS_OK;
+}
+
+template <typename T>
+u32 grid_for(ss_context* c, int H) {
+    switch (H) {
+    case 2: return count_grid<T, 2>(c);
+    case 3: return count_grid<T, 3>(c);
+    case 4: return count_grid<T, 4>(c);
+    case 5: return count_grid<T, 5>(c);
+    case 6: return count_grid<T, 6>(c);
+    case 7: return count_grid<T, 7>(c);
+    case 8: return count_grid<T, 8>(c);
+    case 9: return count_grid<T, 9>(c);
+    default: return count_grid<T, 10>(c);
+    }
+}
+
+template <typename T>
+size_t k1_smem(int s, u32 B) {
+    typedef typename Traits<T>::Key K;
+    return (size_t)std::max<u32>((u32)s, B) * sizeof(K);
+}
+
+template <typename T>
+ss_status set_k1_attrs(ss_context* c) {
+    typedef typename Traits<T>::Key K;
+    CK(cudaFuncSetAttribute(sample_tree_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)(16384 * sizeof(K))));
+    CK(cudaFuncSetAttribute(tree_from_keys_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)(16384 * sizeof(K))));
+    return SS_OK;
+}
+
+ss_status ensure_small(ss_context* c) {
+    if (c->d_ctl) return SS_OK;
+    CK(cudaMalloc(&c->d_ctl, sizeof(LevelCtl) * (SS_MAX_LEVELS + 1)));
+    CK(cudaMalloc(&c->d_res, sizeof(SelectResult)));
+    CK(cudaMalloc(&c->d_totals, sizeof(u64) * SS_MAX_LEVELS * MAX_B));
+    CK(cudaMalloc(&c->d_cta_counts, sizeof(u32) * (size_t)MAX_GRID * MAX_B));
+    CK(cudaMalloc(&c->d_offsets, sizeof(u64) * MAX_GRID));
+    CK(cudaMalloc(&c->d_tree, sizeof(u64) * SS_MAX_LEVELS * MAX_B));
+    CK(cudaMalloc(&c->d_spl, sizeof(u64) * SS_MAX_LEVELS * MAX_B));
+    CK(cudaMalloc(&c->d_eq, (size_t)SS_MAX_LEVELS * MAX_B));
+    CK(cudaMallocHost(&c->h_res, sizeof(SelectResult)));
+    return SS_OK;
+}
+
+ss_status prof_init(ss_context* c) {
+    if (c->ev_ready) return SS_OK;
+    for (int l = 0; l < SS_MAX_LEVELS; ++l)
+        for (int q = 0; q < 3; ++q)
+            for (int e = 0; e < 2; ++e) CK(cudaEventCreate(&c->ev[l][q][e]));
+    c->ev_ready = true;
+    return SS_OK;
+}
+
+// Record the start (e=0) / end (e=1) event of kernel q at level l.
+inline void mark(ss_context* c, int l, int q, int e, cudaStream_t st) {
+    if (!c->cfg.profile || l >= SS_MAX_LEVELS) return;
+    cudaEventRecord(c->ev[l][q][e], st);
+    if (e) c->ev_used[l][q] = true;
+}
+
+void prof_collect(ss_context* c) {
+    for (int l = 0; l < SS_MAX_LEVELS; ++l)
+        for (int q = 0; q < 3; ++q) {
+            float ms = 0.f;
+            if (c->cfg.profile && c->ev_used[l][q])
+                cudaEventElapsedTime(&ms, c->ev[l][q][0], c->ev[l][q][1]);
+            c->stats.ms_kernel[l][q] = ms;
+            c->ev_used[l][q] = false;
+        }
+    (void)cudaGetLastError();
+}
+
+int expected_levels(u64 n, int b, u32 B) {
+    // n_{l+1} ~ n_l / b times the size bias of the bucket holding k (~1.1 for
+    // s/b = 16); plan with 1.5x slack, fall back to more levels if needed.
+    int L = 0;
+    double m = (double)n;
+    while (m > (double)B && L < SS_MAX_LEVELS - 2) {
+        m = m * 1.5 / b;
+        ++L;
+    }
+    return L;
+}
+
+template <typename T>
+ss_status launch_k1(ss_context* c, const T* in, int lev, int s, int b, int fixup, u32 B, int final_level,
+                    cudaStream_t st) {
+    typedef typename Traits<T>::Key K;
+    K* tree = reinterpret_cast<K*>(c->d_tree) + (size_t)lev * MAX_B;
+    K* spl = reinterpret_cast<K*>(c->d_spl) + (size_t)lev * MAX_B;
+    uint8_t* eq = c->d_eq + (size_t)lev * MAX_B;
+    mark(c, lev, 0, 0, st);
+    sample_tree_kernel<T><<<1, K1_THREADS, k1_smem<T>(s, B), st>>>(
+        in, c->d_ctl + lev, c->d_res, tree, spl, eq, s, b, fixup, B, c->cfg.seed, lev, final_level);
+    CKLAUNCH("sample_tree_kernel");
+    mark(c, lev, 0, 1, st);
+    ++c->launches;
+    return SS_OK;
+}
+
+template <typename T>
+ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cudaStream_t st) {
+    typedef typename Traits<T>::Key K;
+    const int b = c->cfg.b_exact, H = log2i(b), s = sample_size(c->cfg, b);
+    const u32 B = (u32)c->cfg.base_case;
+    ss_status rc;
+    if ((rc = ensure_small(c))) return rc;
+    if (c->cfg.profile && (rc = prof_init(c))) return rc;
+    c->launches = 0;
+    c->d2h = 0;
+    if ((rc = grow(c, (void**)&c->d_oracles, &c->cap_oracles, n + 64))) return rc;
+    // survivor ping-pong buffers: a level's survivors never exceed its input
+    for (int i = 0; i < 2; ++i)
+        if ((rc = grow(c, &c->d_buf[i], &c->cap_buf[i], n * sizeof(T)))) return rc;
+    init_kernel<<<1, 1024, 0, st>>>(c->d_ctl, SS_MAX_LEVELS + 1, c->d_totals, SS_MAX_LEVELS * MAX_B, c->d_res,
+                                    n, k);
+    CKLAUNCH("init_kernel");
+    ++c->launches;
+    const u32 grid = grid_for<T>(c, H);
+    int L = expected_levels(n, b, B);
+    int lev = 0;
+    const T* in = d;
+    for (;;) {
+        for (; lev < L; ++lev) {
+            if ((rc = launch_k1<T>(c, in, lev, s, b, 1, B, 0, st))) return rc;
+            CountArgs a{};
+            a.ctl = c->d_ctl + lev;
+            a.ctl_next = c->d_ctl + lev + 1;
+            a.res = c->d_res;
+            a.tree = reinterpret_cast<K*>(c->d_tree) + (size_t)lev * MAX_B;
+            a.spl = reinterpret_cast<K*>(c->d_spl) + (size_t)lev * MAX_B;
+            a.eq = c->d_eq + (size_t)lev * MAX_B;
+            a.oracles = c->d_oracles;
+            a.cta_counts = c->d_cta_counts;
+            a.totals = c->d_totals + (size_t)lev * MAX_B;
+            a.offsets = c->d_offsets;
+            a.level = lev;
+            a.tail = TAIL_EXACT;
+            mark(c, lev, 1, 0, st);
+            if ((rc = launch_count<T>(c, H, in, a, st))) return rc;
+            mark(c, lev, 1, 1, st);
+            ++c->launches;
+            if (a.grid != grid) return fail(c, SS_ERR_INTERNAL, "grid mismatch");
+            T* out = reinterpret_cast<T*>(c->d_buf[lev & 1]);
+            FilterArgs f{};
+            f.ctl = c->d_ctl + lev;
+            f.res = c->d_res;
+            f.oracles = c->d_oracles;
+            f.offsets = c->d_offsets;
+            f.grid = grid;
+            mark(c, lev, 2, 0, st);
+            filter_kernel<T><<<grid, K5_THREADS, 0, st>>>(in, out, f);
+            CKLAUNCH("filter_kernel");
+            mark(c, lev, 2, 1, st);
+            ++c->launches;
+            in = out;
+        }
+        if ((rc = launch_k1<T>(c, in, lev, s, b, 1, B, 1, st))) return rc;
+        CK(cudaMemcpyAsync(c->h_res, c->d_res, sizeof(SelectResult), cudaMemcpyDeviceToHost, st));
+        c->d2h += sizeof(SelectResult);
+        CK(cudaStreamSynchronize(st));
+        if (c->h_res->done) break;
+        if (!c->h_res->incomplete || lev >= SS_MAX_LEVELS - 2)
+            return fail(c, SS_ERR_INTERNAL, "recursion did not terminate");
+        CK(cudaMemsetAsync(&c->d_res->incomplete, 0, sizeof(int), st));
+        L = lev + 1;
+    }
+    const SelectResult& r = *c->h_res;
+    std::memcpy(h_result, &r.bits, sizeof(T));
+    ss_stats& S = c->stats;
+    std::memset(&S, 0, sizeof(S));
+    S.levels = r.levels;
+    S.equality_exit = r.eq_exit;
+    double bytes = 0;
+    const double Sz = (double)sizeof(T);
+    for (int l = 0; l <= r.levels && l < SS_MAX_LEVELS; ++l) {
+        S.n_level[l] = r.n_level[l];
+        S.bucket[l] = r.bucket[l];
+    }
+    for (int l = 0; l < r.levels; ++l) {
+        double nl = (double)r.n_level[l];
+        bytes += Sz * nl + nl;                          // count: read + oracle write
+        bool filtered = !(r.eq_exit && l == r.levels - 1);
+        if (filtered) bytes += nl + 2.0 * Sz * (double)r.n_level[l + 1];  // oracle read + gather + write
+    }
+    if (!r.eq_exit) bytes += Sz * (double)r.n_level[r.levels];  // base case reads its input
+    S.bytes_algorithmic = bytes;
+    S.launches = c->launches;
+    S.h2d_bytes = c->h2d;
+    S.d2h_bytes = c->d2h;
+    prof_collect(c);
+    return SS_OK;
+}
+
+template <typename T>
+ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_result, int64_t* h_rank,
+                     cudaStream_t st) {
+    typedef typename Traits<T>::Key K;
+    const int H = log2i(b);
+    const int s = c->cfg.sample_size > 0 ? c->cfg.sample_size : sample_size(c->cfg, b);
+    if (s < b) return fail(c, SS_ERR_INVALID_ARGUMENT, "sample_size must be >= b");
+    ss_status rc;
+    if ((rc = ensure_small(c))) return rc;
+    if (c->cfg.profile && (rc = prof_init(c))) return rc;
+    c->launches = 0;
+    c->d2h = 0;
+    init_kernel<<<1, 1024, 0, st>>>(c->d_ctl, 2, c->d_totals, MAX_B, c->d_res, n, k);
+    CKLAUNCH("init_kernel");
+    ++c->launches;
+    if ((rc = launch_k1<T>(c, d, 0, s, b, 0, 0, 0, st))) return rc;
+    CountArgs a{};
+    a.ctl = c->d_ctl;
+    a.ctl_next = c->d_ctl + 1;
+    a.res = c->d_res;
+    a.tree = reinterpret_cast<K*>(c->d_tree);
+    a.spl = reinterpret_cast<K*>(c->d_spl);
+    a.eq = c->d_eq;
+    a.oracles = nullptr;
+    a.cta_counts = nullptr;
+    a.totals = c->d_totals;
+    a.offsets = nullptr;
+    a.level = 0;
+    a.tail = TAIL_APPROX;
+    mark(c, 0, 1, 0, st);
+    if ((rc = launch_count<T>(c, H, d, a, st))) return rc;
+    mark(c, 0, 1, 1, st);
+    ++c->launches;
+    CK(cudaMemcpyAsync(c->h_res, c->d_res, sizeof(SelectResult), cudaMemcpyDeviceToHost, st));
+    c->d2h += sizeof(SelectResult);
+    CK(cudaStreamSynchronize(st));
+    const SelectResult& r = *c->h_res;
+    if (!r.done) return fail(c, SS_ERR_INTERNAL, "approximate select produced no result");
+    std::memcpy(h_result, &r.bits, sizeof(T));
+    if (h_rank) *h_rank = r.rank;
+    ss_stats& S = c->stats;
+    std::memset(&S, 0, sizeof(S));
+    S.levels = 1;
+    S.n_level[0] = (int64_t)n;
+    S.bucket[0] = (int32_t)r.split_index;
+    S.bytes_algorithmic = (double)sizeof(T) * (double)n;
+    S.launches = c->launches;
+    S.h2d_bytes = c->h2d;
+    S.d2h_bytes = c->d2h;
+    prof_collect(c);
+    return SS_OK;
+}
+
+ss_status check_common(ss_context* c, ss_dtype dt, const void* p, int64_t n, int64_t k, void* out) {
+    if (!c) return SS_ERR_INVALID_ARGUMENT;
+    if (!dt_size(dt)) return fail(c, SS_ERR_INVALID_ARGUMENT, "unknown dtype");
+    if (!p || !out) return fail(c, SS_ERR_INVALID_ARGUMENT, "NULL pointer");
+    if (n < 1) return fail(c, SS_ERR_INVALID_ARGUMENT, "n must be >= 1");
+    if (k < 0 || k >= n) return fail(c, SS_ERR_INVALID_ARGUMENT, "k must be in [0, n)");
+    if (((uintptr_t)p) % dt_size(dt)) return fail(c, SS_ERR_INVALID_ARGUMENT, "data not naturally aligned");
+    return SS_OK;
+}
+
+template <typename F>
+ss_status dispatch(ss_dtype dt, F&& f) {
+    switch (dt) {
+    case SS_FLOAT32: return f((float*)nullptr);
+    case SS_FLOAT64: return f((double*)nullptr);
+    case SS_INT32: return f((int*)nullptr);
+    case SS_INT64: return f((long long*)nullptr);
+    default: return SS_ERR_INVALID_ARGUMENT;
+    }
+}
+
+ss_status stage_host(ss_context* c, const void* h, size_t bytes, cudaStream_t st) {
+    ss_status rc = grow(c, &c->d_stage, &c->cap_stage, bytes);
+    if (rc) return rc;
+    CK(cudaMemcpyAsync(c->d_stage, h, bytes, cudaMemcpyHostToDevice, st));
+    c->h2d = (int64_t)bytes;
+    return SS_OK;
+}
+
+}  // namespace
+
+// =========================================================== C ABI ========
+extern "C" {
+
+int ss_abi_version(void) { return SS_ABI_VERSION; }
+
+const char* ss_status_string(ss_status s) {
+    switch (s) {
+    case SS_OK: return "SS_OK";
+    case SS_ERR_INVALID_ARGUMENT: return "SS_ERR_INVALID_ARGUMENT";
+    case SS_ERR_CUDA: return "SS_ERR_CUDA";
+    case SS_ERR_OUT_OF_MEMORY: return "SS_ERR_OUT_OF_MEMORY";
+    case SS_ERR_INTERNAL: return "SS_ERR_INTERNAL";
+    default: return "SS_UNKNOWN_STATUS";
+    }
+}
+
+ss_status ss_create(int device, ss_context** out) {
+    if (!out || device < 0) return SS_ERR_INVALID_ARGUMENT;
+    *out = nullptr;
+    int ndev = 0;
+    if (cudaGetDeviceCount(&ndev) != cudaSuccess || device >= ndev) {
+        (void)cudaGetLastError();
+        return SS_ERR_CUDA;
+    }
+    ss_context* c = new (std::nothrow) ss_context();
+    if (!c) return SS_ERR_OUT_OF_MEMORY;
+    c->device = device;
+    c->cfg.b_exact = 256;
+    c->cfg.sample_size = 0;
+    c->cfg.base_case = 16384;
+    c->cfg.ctas_per_sm = 4;
+    c->cfg.profile = 0;
+    c->cfg.seed = 0x5A17;
+    DevGuard g(device);
+    if (cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess) {
+        (void)cudaGetLastError();
+        delete c;
+        return SS_ERR_CUDA;
+    }
+    ss_status rc = ensure_small(c);
+    if (!rc) rc = set_k1_attrs<float>(c);
+    if (!rc) rc = set_k1_attrs<double>(c);
+    if (!rc) rc = set_k1_attrs<int>(c);
+    if (!rc) rc = set_k1_attrs<long long>(c);
+    if (rc) {
+        ss_destroy(c);
+        return rc;
+    }
+    *out = c;
+    return SS_OK;
+}
+
+void ss_destroy(ss_context* c) {
+    if (!c) return;
+    DevGuard g(c->device);
+    cudaFree(c->d_oracles);
+    cudaFree(c->d_buf[0]);
+    cudaFree(c->d_buf[1]);
+    cudaFree(c->d_stage);
+    cudaFree(c->d_ctl);
+    cudaFree(c->d_res);
+    cudaFree(c->d_totals);
+    cudaFree(c->d_cta_counts);
+    cudaFree(c->d_offsets);
+    cudaFree(c->d_tree);
+    cudaFree(c->d_spl);
+    cudaFree(c->d_eq);
+    if (c->h_res) cudaFreeHost(c->h_res);
+    if (c->ev_ready)
+        for (int l = 0; l < SS_MAX_LEVELS; ++l)
+            for (int q = 0; q < 3; ++q)
+                for (int e = 0; e < 2; ++e) cudaEventDestroy(c->ev[l][q][e]);
+    (void)cudaGetLastError();
+    delete c;
+}
+
+ss_status ss_get_config(const ss_context* c, ss_config* out) {
+    if (!c || !out) return SS_ERR_INVALID_ARGUMENT;
+    *out = c->cfg;
+    return SS_OK;
+}
+
+ss_status ss_set_config(ss_context* c, const ss_config* cfg) {
+    if (!c || !cfg) return SS_ERR_INVALID_ARGUMENT;
+    if (!pow2(cfg->b_exact) || cfg->b_exact < 4 || cfg->b_exact > 256)
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "b_exact must be a power of two in [4, 256]");
+    if (cfg->sample_size != 0 && (!pow2(cfg->sample_size) || cfg->sample_size > 16384 ||
+                                  cfg->sample_size < cfg->b_exact))
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "sample_size must be 0 or a power of two in [b, 16384]");
+    if (!pow2(cfg->base_case) || cfg->base_case < 256 || cfg->base_case > 16384)
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "base_case must be a power of two in [256, 16384]");
+    if (cfg->profile != 0 && cfg->profile != 1)
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "profile must be 0 or 1");
+    if (cfg->ctas_per_sm < 1 || cfg->ctas_per_sm > 16)
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "ctas_per_sm must be in [1, 16]");
+    c->cfg = *cfg;
+    return SS_OK;
+}
+
+ss_status ss_last_stats(const ss_context* c, ss_stats* out) {
+    if (!c || !out) return SS_ERR_INVALID_ARGUMENT;
+    *out = c->stats;
+    return SS_OK;
+}
+
+const char* ss_last_error(const ss_context* c) { return c ? c->err.c_str() : "NULL context"; }
+
+static ss_status select_impl(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k,
+                             void* h_result, void* stream);
+
+ss_status ss_select(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k, void* h_result,
+                    void* stream) {
+    if (c) c->h2d = 0;
+    return select_impl(c, dt, d_data, n, k, h_result, stream);
+}
+
+static ss_status select_impl(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k,
+                             void* h_result, void* stream) {
+    ss_status rc = check_common(c, dt, d_data, n, k, h_result);
+    if (rc) return rc;
+    DevGuard g(c->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    try {
+        return dispatch(dt, [&](auto* tag) {
+            typedef std::remove_pointer_t<decltype(tag)> T;
+            return run_exact<T>(c, (const T*)d_data, (u64)n, (u64)k, h_result, st);
+        });
+    } catch (...) {
+        return fail(c, SS_ERR_INTERNAL, "exception in ss_select");
+    }
+}
+
+ss_status ss_select_host(ss_context* c, ss_dtype dt, const void* h_data, int64_t n, int64_t k,
+                         void* h_result, void* stream) {
+    ss_status rc = check_common(c, dt, h_data, n, k, h_result);
+    if (rc) return rc;
+    DevGuard g(c->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    if ((rc = stage_host(c, h_data, (size_t)n * dt_size(dt), st))) return rc;
+    return select_impl(c, dt, c->d_stage, n, k, h_result, stream);
+}
+
+static ss_status approx_impl(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k, int32_t b,
+                             void* h_result, int64_t* h_rank, void* stream);
+
+ss_status ss_approx_select(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k, int32_t b,
+                           void* h_result, int64_t* h_rank, void* stream) {
+    if (c) c->h2d = 0;
+    return approx_impl(c, dt, d_data, n, k, b, h_result, h_rank, stream);
+}
+
+static ss_status approx_impl(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k, int32_t b,
+                             void* h_result, int64_t* h_rank, void* stream) {
+    ss_status rc = check_common(c, dt, d_data, n, k, h_result);
+    if (rc) return rc;
+    if (!pow2(b) || b < 4 || b > 1024) return fail(c, SS_ERR_INVALID_ARGUMENT, "b must be a power of two in [4, 1024]");
+    DevGuard g(c->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    try {
+        return dispatch(dt, [&](auto* tag) {
+            typedef std::remove_pointer_t<decltype(tag)> T;
+            return run_approx<T>(c, (const T*)d_data, (u64)n, (u64)k, b, h_result, h_rank, st);
+        });
+    } catch (...) {
+        return fail(c, SS_ERR_INTERNAL, "exception in ss_approx_select");
+    }
+}
+
+ss_status ss_approx_select_host(ss_context* c, ss_dtype dt, const void* h_data, int64_t n, int64_t k,
+                                int32_t b, void* h_result, int64_t* h_rank, void* stream) {
+    ss_status rc = check_common(c, dt, h_data, n, k, h_result);
+    if (rc) return rc;
+    DevGuard g(c->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    if ((rc = stage_host(c, h_data, (size_t)n * dt_size(dt), st))) return rc;
+    return approx_impl(c, dt, c->d_stage, n, k, b, h_result, h_rank, stream);
+}
+
+// ------------------------------------------------------------- steps ------
+ss_status ss_step_sample(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int32_t level,
+                         int64_t slot_begin, int64_t count, void* d_sample_keys, void* stream) {
+    if (!c || !dt_size(dt) || !d_data || !d_sample_keys || n < 1 || count < 0 || slot_begin < 0 || level < 0)
+        return c ? fail(c, SS_ERR_INVALID_ARGUMENT, "ss_step_sample: bad argument") : SS_ERR_INVALID_ARGUMENT;
+    if (count == 0) return SS_OK;
+    DevGuard g(c->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    return dispatch(dt, [&](auto* tag) -> ss_status {
+        typedef std::remove_pointer_t<decltype(tag)> T;
+        typedef typename Traits<T>::Key K;
+        u32 blocks = (u32)std::min<int64_t>((count + 255) / 256, 1024);
+        sample_keys_kernel<T><<<blocks, 256, 0, st>>>((const T*)d_data, (u64)n, level, (u64)slot_begin,
+                                                      (u64)count, c->cfg.seed, (K*)d_sample_keys);
+        CKLAUNCH("sample_keys_kernel");
+        return SS_OK;
+    });
+}
+
+ss_status ss_step_tree(ss_context* c, ss_dtype dt, const void* d_sample_keys, int32_t s, int32_t b,
+                       int32_t fixup, void* d_tree, void* d_splitters, uint8_t* d_eq, void* stream) {
+    if (!c || !dt_size(dt) || !d_sample_keys || !d_tree || !pow2(s) || s > 16384 || !pow2(b) || b < 2 ||
+        b > 1024 || s < b)
+        return c ? fail(c, SS_ERR_INVALID_ARGUMENT, "ss_step_tree: bad argument") : SS_ERR_INVALID_ARGUMENT;
+    DevGuard g(c->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    if (dt_size(dt) == 4) {
+        tree_from_keys_kernel<u32><<<1, K1_THREADS, (size_t)s * 4, st>>>(
+            (const u32*)d_sample_keys, s, b, fixup, (u32*)d_tree, (u32*)d_splitters, d_eq);
+    } else {
+        tree_from_keys_kernel<u64><<<1, K1_THREADS, (size_t)s * 8, st>>>(
+            (const u64*)d_sample_keys, s, b, fixup, (u64*)d_tree, (u64*)d_splitters, d_eq);
+    }
+    CKLAUNCH("tree_from_keys_kernel");
+    return SS_OK;
+}
+
+ss_status ss_step_count(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, const void* d_tree,
+                        int32_t b, uint64_t* d_totals, uint8_t* d_oracles, void* stream) {
+    if (!c || !dt_size(dt) || !d_data || !d_tree || !d_totals || n < 1 || !pow2(b) || b < 4 || b > 1024 ||
+        (d_oracles && b > 256) || ((uintptr_t)d_data) % dt_size(dt))
+        return c ? fail(c, SS_ERR_INVALID_ARGUMENT, "ss_step_count: bad argument") : SS_ERR_INVALID_ARGUMENT;
+    DevGuard g(c->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    ss_status rc = ensure_small(c);
+    if (rc) return rc;
+    CK(cudaMemsetAsync(d_totals, 0, sizeof(u64) * b, st));
+    return dispatch(dt, [&](auto* tag) -> ss_status {
+        typedef std::remove_pointer_t<decltype(tag)> T;
+        CountArgs a{};
+        a.tree = d_tree;
+        a.oracles = d_oracles;
+        a.cta_counts = c->d_cta_counts;
+        a.totals = (u64*)d_totals;
+        a.n = (u64)n;
+        a.tail = TAIL_NONE;
+        ss_status r2 = launch_count<T>(c, log2i(b), (const T*)d_data, a, st);
+        if (r2) return r2;
+        c->step_ptr = d_data;
+        c->step_n = (u64)n;
+        c->step_b = b;
+        c->step_dt = (int)dt;
+        c->step_grid = a.grid;
+        return SS_OK;
+    });
+}
+
+ss_status ss_step_filter(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, const uint8_t* d_oracles,
+                         int32_t bucket, void* d_out, uint64_t* d_count, void* stream) {
+    if (!c || !dt_size(dt) || !d_data || !d_oracles || !d_out || !d_count || n < 1 || bucket < 0)
+        return c ? fail(c, SS_ERR_INVALID_ARGUMENT, "ss_step_filter: bad argument") : SS_ERR_INVALID_ARGUMENT;
+    if (c->step_ptr != d_data || c->step_n != (u64)n || c->step_dt != (int)dt || bucket >= c->step_b)
+        return fail(c, SS_ERR_INVALID_ARGUMENT,
+                    "ss_step_filter must follow ss_step_count on the same data (per-CTA counts)");
+    DevGuard g(c->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    const u32 grid = c->step_grid;
+    return dispatch(dt, [&](auto* tag) -> ss_status {
+        typedef std::remove_pointer_t<decltype(tag)> T;
+        Chunking ch = make_chunking((const T*)d_data, (u64)n, grid, Group<T>::vecs);
+        offsets_kernel<<<1, 1024, 0, st>>>(c->d_cta_counts, (u32)c->step_b, (u32)bucket, ch.ncta, c->d_offsets);
+        CKLAUNCH("offsets_kernel");
+        CK(cudaMemsetAsync(d_count, 0, sizeof(u64), st));
+        FilterArgs f{};
+        f.oracles = d_oracles;
+        f.offsets = c->d_offsets;
+        f.count_out = (u64*)d_count;
+        f.n = (u64)n;
+        f.bucket = (u32)bucket;
+        f.grid = grid;
+        filter_kernel<T><<<grid, K5_THREADS, 0, st>>>((const T*)d_data, (T*)d_out, f);
+        CKLAUNCH("filter_kernel");
+        return SS_OK;
+    });
+}
+
+ss_status ss_step_search(ss_context* c, const uint64_t* d_totals, int32_t b, int64_t k, const uint8_t* d_eq,
+                         int64_t* d_out, void* stream) {
+    if (!c || !d_totals || !d_out || b < 1 || b > 1024 || k < 0)
+        return c ? fail(c, SS_ERR_INVALID_ARGUMENT, "ss_step_search: bad argument") : SS_ERR_INVALID_ARGUMENT;
+    DevGuard g(c->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    search_kernel<<<1, 256, 0, st>>>((const u64*)d_totals, (u32)b, (u64)k, d_eq, (long long*)d_out);
+    CKLAUNCH("search_kernel");
+    return SS_OK;
+}
+
+ss_status ss_step_keys_to_values(ss_context* c, ss_dtype dt, const void* d_keys, int64_t count, void* d_values,
+                                 void* stream) {
+    if (!c || !dt_size(dt) || !d_keys || !d_values || count < 0)
+        return c ? fail(c, SS_ERR_INVALID_ARGUMENT, "ss_step_keys_to_values: bad argument") : SS_ERR_INVALID_ARGUMENT;
+    if (count == 0) return SS_OK;
+    DevGuard g(c->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    u32 blocks = (u32)std::min<int64_t>((count + 255) / 256, 4096);
+    return dispatch(dt, [&](auto* tag) -> ss_status {
+        typedef std::remove_pointer_t<decltype(tag)> T;
+        typedef typename Traits<T>::Key K;
+        keys_to_values_kernel<T><<<blocks, 256, 0, st>>>((const K*)d_keys, (u64)count, (K*)d_values);
+        CKLAUNCH("keys_to_values_kernel");
+        return SS_OK;
+    });
+}
+
+}  // extern "C"
