@@ -81,14 +81,13 @@ class ClockSampler:
         try:
             import pynvml
             pynvml.nvmlInit()
-            # CUDA_VISIBLE_DEVICES remaps indices; match by PCI bus id
+            # CUDA_VISIBLE_DEVICES remaps indices; match by UUID
             import torch
-            bus = torch.cuda.get_device_properties(device).pci_bus_id \
-                if hasattr(torch.cuda.get_device_properties(device), "pci_bus_id") else None
             h = None
-            if bus is not None:
+            uuid = getattr(torch.cuda.get_device_properties(device), "uuid", None)
+            if uuid is not None:
                 try:
-                    h = pynvml.nvmlDeviceGetHandleByPciBusId(bus)
+                    h = pynvml.nvmlDeviceGetHandleByUUID(("GPU-" + str(uuid)).encode())
                 except Exception:
                     h = None
             if h is None:
