@@ -82,35 +82,38 @@ struct SelectResult {
 };
 
 // ------------------------------------------------------------ chunking ----
-// Element -> CTA mapping shared by the count (K2) and filter (K5) kernels;
-// the filter must see exactly the count's per-CTA ranges so that the K3
-// offsets apply (§IV.G).  Elements [0, head) are peeled so that the
-// vector body starts 16-byte aligned; the body is nvec 16-byte vectors of
-// V = 16/sizeof(T) elements; [tail_begin, n) is the ragged tail.  CTA g owns
-// body vectors [g*vpc, min((g+1)*vpc, nvec)); CTA 0 also owns the head, the
-// last active CTA the tail.
+// Element -> unit mapping shared by the count (K2) and filter (K5) kernels;
+// the filter must see exactly the count's partition so that the K3 offsets
+// apply (§IV.G).  The body is cut into 16-element groups (16 oracle
+// bytes = one 128-bit load); a "unit" is the contiguous run of groups owned
+// by one warp: unit u = g * UNIT_WARPS + w owns groups [u*gpw, (u+1)*gpw).
+// Elements [0, head) are peeled so the body starts 16-byte aligned (unit 0
+// owns them); [tail_begin, n) (< 16 elements) belongs to the last unit of the
+// last active CTA.  K2 counts per unit; K5 compacts per unit with no
+// cross-warp synchronisation.
+constexpr u32 UNIT_WARPS = 16;          // warps per CTA in K2 and K5 (512 threads)
+constexpr u64 MIN_GROUPS_PER_UNIT = 4;  // 64 elements
+
 struct Chunking {
-    u64 head, nvec, tail_begin, vpc;
+    u64 head, ngroups, tail_begin, gpw;
     u32 ncta;
 };
 
 template <typename T>
-__host__ __device__ __forceinline__ Chunking make_chunking(const T* p, u64 n, u32 grid, u32 group_vecs) {
-    const u64 V = 16 / sizeof(T);
+__host__ __device__ __forceinline__ Chunking make_chunking(const T* p, u64 n, u32 grid) {
     Chunking c;
     u64 mis = (u64)((uintptr_t)p & 15u);
     u64 head = mis ? (16 - mis) / sizeof(T) : 0;
     if (head > n) head = n;
     c.head = head;
-    c.nvec = (n - head) / V;
-    c.tail_begin = head + c.nvec * V;
-    // at least 16 groups per CTA so tiny levels use few CTAs
-    u64 min_vpc = (u64)group_vecs * 16;
-    u64 want = (c.nvec + grid - 1) / grid;
-    if (want < min_vpc) want = min_vpc;
-    want = (want + group_vecs - 1) / group_vecs * group_vecs;
-    c.vpc = want;
-    u64 nc = (c.nvec + want - 1) / want;
+    c.ngroups = (n - head) / 16;
+    c.tail_begin = head + c.ngroups * 16;
+    const u64 units_max = (u64)grid * UNIT_WARPS;
+    u64 gpw = (c.ngroups + units_max - 1) / units_max;
+    if (gpw < MIN_GROUPS_PER_UNIT) gpw = MIN_GROUPS_PER_UNIT;
+    c.gpw = gpw;
+    const u64 units = (c.ngroups + gpw - 1) / gpw;
+    u64 nc = (units + UNIT_WARPS - 1) / UNIT_WARPS;
     if (nc == 0) nc = 1;
     if (nc > grid) nc = grid;
     c.ncta = (u32)nc;

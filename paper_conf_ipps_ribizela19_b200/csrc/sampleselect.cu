@@ -35,6 +35,7 @@ struct ss_context {
     SelectResult* d_res = nullptr;
     u64* d_totals = nullptr;     // [SS_MAX_LEVELS][MAX_B]
     u32* d_cta_counts = nullptr; // [MAX_GRID][MAX_B]
+    u32* d_warp_counts = nullptr; // [MAX_GRID][UNIT_WARPS][256]
     u64* d_offsets = nullptr;    // [MAX_GRID]
     u64* d_tree = nullptr;       // [SS_MAX_LEVELS][MAX_B] keys (u32 keys use the same bytes)
     u64* d_spl = nullptr;
@@ -54,7 +55,7 @@ struct ss_context {
     int64_t h2d = 0, d2h = 0;   // bytes copied by the current call
 };
 
-static constexpr u32 MAX_GRID = 4096;
+static constexpr u32 MAX_GRID = 2048;
 
 namespace {
 
@@ -126,7 +127,11 @@ u32 count_grid(ss_context* c) {
     int dev = c->device & 63;
     if (!occ[dev]) {
         int o = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, count_kernel<T, H>, K2_THREADS, 0);
+        typedef typename Traits<T>::Key K;
+        cudaFuncSetAttribute(count_kernel<T, H>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                             (int)count_smem_bytes<H, K>());
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, count_kernel<T, H>, K2_THREADS,
+                                                      count_smem_bytes<H, K>());
         occ[dev] = o > 0 ? o : 1;
     }
     u32 per = (u32)std::max(1, std::min(c->cfg.ctas_per_sm, occ[dev]));
@@ -138,7 +143,8 @@ ss_status launch_count(ss_context* c, int H, const T* in, CountArgs& a, cudaStre
 #define SS_COUNT_CASE(h)                                                     \
     case h:                                                                  \
         a.grid = count_grid<T, h>(c);                                        \
-        count_kernel<T, h><<<a.grid, K2_THREADS, 0, st>>>(in, a);            \
+        count_kernel<T, h><<<a.grid, K2_THREADS,                             \
+            count_smem_bytes<h, typename Traits<T>::Key>(), st>>>(in, a);    \
         break;
     switch (H) {
         SS_COUNT_CASE(2) SS_COUNT_CASE(3) SS_COUNT_CASE(4) SS_COUNT_CASE(5) SS_COUNT_CASE(6)
@@ -178,6 +184,7 @@ ss_status set_k1_attrs(ss_context* c) {
                             (int)(16384 * sizeof(K))));
     CK(cudaFuncSetAttribute(tree_from_keys_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                             (int)(16384 * sizeof(K))));
+    CK(cudaFuncSetAttribute(filter_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)FILTER_SMEM));
     return SS_OK;
 }
 
@@ -187,6 +194,7 @@ ss_status ensure_small(ss_context* c) {
     CK(cudaMalloc(&c->d_res, sizeof(SelectResult)));
     CK(cudaMalloc(&c->d_totals, sizeof(u64) * SS_MAX_LEVELS * MAX_B));
     CK(cudaMalloc(&c->d_cta_counts, sizeof(u32) * (size_t)MAX_GRID * MAX_B));
+    CK(cudaMalloc(&c->d_warp_counts, sizeof(u32) * (size_t)MAX_GRID * UNIT_WARPS * 256));
     CK(cudaMalloc(&c->d_offsets, sizeof(u64) * MAX_GRID));
     CK(cudaMalloc(&c->d_tree, sizeof(u64) * SS_MAX_LEVELS * MAX_B));
     CK(cudaMalloc(&c->d_spl, sizeof(u64) * SS_MAX_LEVELS * MAX_B));
@@ -285,6 +293,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             a.eq = c->d_eq + (size_t)lev * MAX_B;
             a.oracles = c->d_oracles;
             a.cta_counts = c->d_cta_counts;
+            a.warp_counts = c->d_warp_counts;
             a.totals = c->d_totals + (size_t)lev * MAX_B;
             a.offsets = c->d_offsets;
             a.level = lev;
@@ -300,9 +309,11 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             f.res = c->d_res;
             f.oracles = c->d_oracles;
             f.offsets = c->d_offsets;
+            f.warp_counts = c->d_warp_counts;
+            f.b_count = (u32)b;
             f.grid = grid;
             mark(c, lev, 2, 0, st);
-            filter_kernel<T><<<grid, K5_THREADS, 0, st>>>(in, out, f);
+            filter_kernel<T><<<grid, K5_THREADS, FILTER_SMEM, st>>>(in, out, f);
             CKLAUNCH("filter_kernel");
             mark(c, lev, 2, 1, st);
             ++c->launches;
@@ -492,6 +503,7 @@ void ss_destroy(ss_context* c) {
     cudaFree(c->d_res);
     cudaFree(c->d_totals);
     cudaFree(c->d_cta_counts);
+    cudaFree(c->d_warp_counts);
     cudaFree(c->d_offsets);
     cudaFree(c->d_tree);
     cudaFree(c->d_spl);
@@ -660,6 +672,7 @@ ss_status ss_step_count(ss_context* c, ss_dtype dt, const void* d_data, int64_t 
         a.tree = d_tree;
         a.oracles = d_oracles;
         a.cta_counts = c->d_cta_counts;
+        a.warp_counts = b <= 256 ? c->d_warp_counts : nullptr;
         a.totals = (u64*)d_totals;
         a.n = (u64)n;
         a.tail = TAIL_NONE;
@@ -686,18 +699,20 @@ ss_status ss_step_filter(ss_context* c, ss_dtype dt, const void* d_data, int64_t
     const u32 grid = c->step_grid;
     return dispatch(dt, [&](auto* tag) -> ss_status {
         typedef std::remove_pointer_t<decltype(tag)> T;
-        Chunking ch = make_chunking((const T*)d_data, (u64)n, grid, Group<T>::vecs);
+        Chunking ch = make_chunking((const T*)d_data, (u64)n, grid);
         offsets_kernel<<<1, 1024, 0, st>>>(c->d_cta_counts, (u32)c->step_b, (u32)bucket, ch.ncta, c->d_offsets);
         CKLAUNCH("offsets_kernel");
         CK(cudaMemsetAsync(d_count, 0, sizeof(u64), st));
         FilterArgs f{};
         f.oracles = d_oracles;
         f.offsets = c->d_offsets;
+        f.warp_counts = c->d_warp_counts;
+        f.b_count = (u32)c->step_b;
         f.count_out = (u64*)d_count;
         f.n = (u64)n;
         f.bucket = (u32)bucket;
         f.grid = grid;
-        filter_kernel<T><<<grid, K5_THREADS, 0, st>>>((const T*)d_data, (T*)d_out, f);
+        filter_kernel<T><<<grid, K5_THREADS, FILTER_SMEM, st>>>((const T*)d_data, (T*)d_out, f);
         CKLAUNCH("filter_kernel");
         return SS_OK;
     });

@@ -1,0 +1,19 @@
+"""Run a few selections for ncu: `python scripts/profile_one.py [log2n] [mode] [b]`."""
+import os, sys
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np, torch
+import datagen
+import paper_conf_ipps_ribizela19_b200 as ss
+log2n = int(sys.argv[1]) if len(sys.argv) > 1 else 28
+mode = sys.argv[2] if len(sys.argv) > 2 else "exact"
+b = int(sys.argv[3]) if len(sys.argv) > 3 else (256 if mode == "exact" else 1024)
+n = 1 << log2n
+x = torch.from_numpy(datagen.uniform(n, np.float32, seed=datagen.dataset_seed(5, 0))).cuda()
+ctx = ss.Context(0)
+for _ in range(3):
+    if mode == "exact":
+        ctx.configure(b_exact=b); v = ctx.select(x, n // 2)
+    else:
+        v = ctx.approx_select(x, n // 2, b)
+torch.cuda.synchronize()
+print(v, ctx.stats())
