@@ -248,9 +248,12 @@ def run_ours(args, rank, world, local_rank):
         step(xd)
     torch.cuda.synchronize()
 
-    # ---- timed region (profile events on: per-kernel device times)
-    ctx.configure(profile=1)
-    k2_ms, k5_ms, step_stats = [], [], []
+    # ---- timed region.  profile=2: the library records CUDA events around
+    # the dominant kernel (level-0 count) on the call's stream and accumulates
+    # its device time over the timed calls (read once afterwards, so nothing
+    # but the select calls runs between steps).
+    ctx.configure(profile=2)
+    ctx.profile_totals(reset=True)
     barrier()
     torch.cuda.synchronize()
     ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -258,15 +261,24 @@ def run_ours(args, rank, world, local_rank):
         ev0.record(stream)
         for _ in range(args.steps):
             step(xd)
-            st = ctx.stats()
-            k2_ms.append(st["ms_kernel"][0][1])
-            k5_ms.append(st["ms_kernel"][0][2])
-            step_stats.append(st)
         ev1.record(stream)
         torch.cuda.synchronize()
     barrier()
     ms = ev0.elapsed_time(ev1) / args.steps
+    prof_timed = ctx.profile_totals(reset=True)
+    # per-kernel breakdown (all kernels timed; separate, informational pass)
+    ctx.configure(profile=1)
+    for _ in range(min(args.steps, 10)):
+        step(xd)
+    torch.cuda.synchronize()
+    prof = ctx.profile_totals(reset=True)
+    last = ctx.stats()
     ctx.configure(profile=0)
+
+    def kavg(level, q, pr=None):
+        pr = pr or prof
+        cnt = pr["count"][level][q]
+        return pr["ms_sum"][level][q] / cnt if cnt else 0.0
     if world > 1:
         t = torch.tensor([ms], device=f"cuda:{dev}", dtype=torch.float64)
         torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
@@ -303,7 +315,7 @@ def run_ours(args, rank, world, local_rank):
     peak, peak_src = measured_peak()
     S = np.dtype(args.dtype).itemsize
     k2_bytes = (S + (1 if exact else 0)) * n          # read S*n, write n oracle bytes
-    k2_avg = float(np.mean(k2_ms))
+    k2_avg = kavg(0, 1, prof_timed)
     achieved = k2_bytes / (k2_avg * 1e-3) / 1e9
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -314,8 +326,7 @@ def run_ours(args, rank, world, local_rank):
             traffic = tk
         except Exception:
             traffic = None
-    last = step_stats[-1]
-    path_bytes = float(np.mean([s_["bytes_algorithmic"] for s_ in step_stats]))
+    path_bytes = float(last["bytes_algorithmic"])
     line = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": max(3, args.warmup), "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
@@ -332,10 +343,10 @@ def run_ours(args, rank, world, local_rank):
                           "achieved_gbs": path_bytes / (ms * 1e-3) / 1e9,
                           "frac_of_peak": path_bytes / (ms * 1e-3) / 1e9 / peak,
                           "frac_of_8tbs": path_bytes / (ms * 1e-3) / 8e12},
-        "kernels_ms": {"k2_count_l0": k2_avg, "k5_filter_l0": float(np.mean(k5_ms)),
-                       "levels": last["levels"], "n_level": last["n_level"],
-                       "ms_kernel_last": last["ms_kernel"]},
-        "gpu_launches": int(sum(s_["launches"] for s_ in step_stats)),
+        "kernels_ms": {"avg_per_level": [[kavg(l, q) for q in range(3)] for l in range(last["levels"] + 1)],
+                       "sum_of_kernels": sum(kavg(l, q) for l in range(last["levels"] + 1) for q in range(3)),
+                       "levels": last["levels"], "n_level": last["n_level"]},
+        "gpu_launches": int(prof_timed["launches"]),
         "clocks": clk.summary(),
         "e2e": e2e,
     }

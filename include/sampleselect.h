@@ -62,7 +62,8 @@ typedef struct {
                              power of two in [256, 16384]. default 16384 */
     int32_t ctas_per_sm;  /* count/filter grid = ctas_per_sm * #SMs. default 4 */
     int32_t profile;      /* 1: record CUDA events around every kernel on the call's
-                             stream and report per-kernel device times in ss_stats */
+                             stream and report per-kernel device times in ss_stats;
+                             2: only around the dominant kernel (level-0 count) */
     uint64_t seed;        /* sampling seed (reading R7). default 0x5A17 */
 } ss_config;
 
@@ -88,6 +89,13 @@ ss_status ss_get_config(const ss_context* ctx, ss_config* out);
 ss_status ss_set_config(ss_context* ctx, const ss_config* cfg);
 ss_status ss_last_stats(const ss_context* ctx, ss_stats* out);
 const char* ss_last_error(const ss_context* ctx);
+/* Totals accumulated over all calls since the last reset: per (level, kernel)
+ * device ms summed from the profile events (ms_sum[SS_MAX_LEVELS*3], index
+ * level*3 + kernel, kernel 0 = K1, 1 = K2, 2 = K5) and how many launches each
+ * sum covers (count[SS_MAX_LEVELS*3]); total kernel launches and calls.  Any
+ * output pointer may be NULL.  reset != 0 zeroes the totals after reading. */
+ss_status ss_profile_totals(ss_context* ctx, double* ms_sum, int64_t* count, int64_t* launches,
+                            int64_t* calls, int32_t reset);
 const char* ss_status_string(ss_status s);
 int       ss_abi_version(void);
 

@@ -103,6 +103,19 @@ class Context:
                 "h2d_bytes": s.h2d_bytes, "d2h_bytes": s.d2h_bytes,
                 "ms_kernel": [list(s.ms_kernel[l]) for l in range(L + 1)]}
 
+    def profile_totals(self, reset: bool = False) -> dict:
+        """Per-(level, kernel) device ms summed over calls made with
+        profile=1, launch and call counts since the last reset."""
+        L = _abi.SS_MAX_LEVELS
+        ms = (ctypes.c_double * (3 * L))()
+        cnt = (ctypes.c_int64 * (3 * L))()
+        launches, calls = ctypes.c_int64(), ctypes.c_int64()
+        self._check(self._lib.ss_profile_totals(self._h, ms, cnt, ctypes.byref(launches),
+                                                ctypes.byref(calls), int(reset)))
+        return {"ms_sum": [[ms[l * 3 + q] for q in range(3)] for l in range(L)],
+                "count": [[cnt[l * 3 + q] for q in range(3)] for l in range(L)],
+                "launches": launches.value, "calls": calls.value}
+
     def _args(self, x):
         """-> (dtype code, pointer, n, numpy dtype, on_device)"""
         if _is_tensor(x):

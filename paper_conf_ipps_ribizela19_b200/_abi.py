@@ -10,7 +10,7 @@ import os
 import threading
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libsampleselect.so")
+LIB_PATH = os.environ.get("SS_LIB") or os.path.join(_PKG, "libsampleselect.so")
 
 SS_FLOAT32, SS_FLOAT64, SS_INT32, SS_INT64 = 0, 1, 2, 3
 SS_MAX_LEVELS = 32
@@ -19,7 +19,7 @@ STATUS = {0: "SS_OK", 1: "SS_ERR_INVALID_ARGUMENT", 2: "SS_ERR_CUDA",
 
 # every symbol include/sampleselect.h declares
 EXPORTS = [
-    "ss_create", "ss_destroy", "ss_get_config", "ss_set_config", "ss_last_stats",
+    "ss_create", "ss_destroy", "ss_get_config", "ss_set_config", "ss_last_stats", "ss_profile_totals",
     "ss_last_error", "ss_status_string", "ss_abi_version",
     "ss_select", "ss_select_host", "ss_approx_select", "ss_approx_select_host",
     "ss_step_sample", "ss_step_tree", "ss_step_count", "ss_step_filter",
@@ -73,6 +73,8 @@ def lib() -> ctypes.CDLL:
         L.ss_get_config.argtypes = [vp, ctypes.POINTER(SSConfig)]
         L.ss_set_config.argtypes = [vp, ctypes.POINTER(SSConfig)]
         L.ss_last_stats.argtypes = [vp, ctypes.POINTER(SSStats)]
+        L.ss_profile_totals.argtypes = [vp, ctypes.POINTER(ctypes.c_double), ctypes.POINTER(i64),
+                                        ctypes.POINTER(i64), ctypes.POINTER(i64), i32]
         L.ss_last_error.argtypes = [vp]
         L.ss_last_error.restype = ctypes.c_char_p
         L.ss_status_string.argtypes = [st]

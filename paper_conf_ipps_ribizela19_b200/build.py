@@ -41,17 +41,19 @@ def up_to_date() -> bool:
     return all(os.path.getmtime(p) <= t for p in _deps())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and up_to_date():
+def build(force: bool = False, verbose: bool = False, out: str | None = None) -> str:
+    target = out or LIB
+    if not force and out is None and up_to_date():
         return LIB
-    tmp = LIB + f".tmp{os.getpid()}"
-    cmd = [NVCC, *NVCC_FLAGS, f"-I{INCLUDE}", "-o", tmp, *_sources()]
+    tmp = target + f".tmp{os.getpid()}"
+    extra = os.environ.get("SS_NVCC_EXTRA", "").split()
+    cmd = [NVCC, *NVCC_FLAGS, *extra, f"-I{INCLUDE}", "-o", tmp, *_sources()]
     if verbose:
         cmd.insert(1, "-Xptxas=-v")
         print(" ".join(cmd), flush=True)
     subprocess.check_call(cmd)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, target)
+    return target
 
 
 if __name__ == "__main__":

@@ -9,6 +9,7 @@
 // case (rare: an unlucky sample) more levels are enqueued.  One device->host
 // copy per call returns the answer; there is no per-level host round trip.
 #include <algorithm>
+#include <cstdlib>
 #include <cstdio>
 #include <cstring>
 #include <new>
@@ -51,6 +52,10 @@ struct ss_context {
     cudaEvent_t ev[SS_MAX_LEVELS][3][2] = {};
     bool ev_used[SS_MAX_LEVELS][3] = {};
     bool ev_ready = false;
+    double prof_sum[SS_MAX_LEVELS][3] = {};   // accumulated device ms per (level, kernel)
+    long long prof_cnt[SS_MAX_LEVELS][3] = {};
+    long long launches_total = 0;
+    long long calls_total = 0;
     int launches = 0;
     int64_t h2d = 0, d2h = 0;   // bytes copied by the current call
 };
@@ -130,6 +135,9 @@ u32 count_grid(ss_context* c) {
         typedef typename Traits<T>::Key K;
         cudaFuncSetAttribute(count_kernel<T, H>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)count_smem_bytes<H, K>());
+#ifdef SS_CARVEOUT
+        cudaFuncSetAttribute(count_kernel<T, H>, cudaFuncAttributePreferredSharedMemoryCarveout, SS_CARVEOUT);
+#endif
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, count_kernel<T, H>, K2_THREADS,
                                                       count_smem_bytes<H, K>());
         occ[dev] = o > 0 ? o : 1;
@@ -185,6 +193,12 @@ ss_status set_k1_attrs(ss_context* c) {
     CK(cudaFuncSetAttribute(tree_from_keys_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                             (int)(16384 * sizeof(K))));
     CK(cudaFuncSetAttribute(filter_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)FILTER_SMEM));
+    // one carveout (all shared) for every kernel of the path: no L1/shared
+    // reconfiguration between consecutive kernels
+#ifdef SS_CARVEOUT
+    CK(cudaFuncSetAttribute(sample_tree_kernel<T>, cudaFuncAttributePreferredSharedMemoryCarveout, SS_CARVEOUT));
+    CK(cudaFuncSetAttribute(filter_kernel<T>, cudaFuncAttributePreferredSharedMemoryCarveout, SS_CARVEOUT));
+#endif
     return SS_OK;
 }
 
@@ -215,6 +229,7 @@ ss_status prof_init(ss_context* c) {
 // Record the start (e=0) / end (e=1) event of kernel q at level l.
 inline void mark(ss_context* c, int l, int q, int e, cudaStream_t st) {
     if (!c->cfg.profile || l >= SS_MAX_LEVELS) return;
+    if (c->cfg.profile == 2 && !(l == 0 && q == 1)) return;   // dominant kernel only
     cudaEventRecord(c->ev[l][q][e], st);
     if (e) c->ev_used[l][q] = true;
 }
@@ -226,6 +241,8 @@ void prof_collect(ss_context* c) {
             if (c->cfg.profile && c->ev_used[l][q])
                 cudaEventElapsedTime(&ms, c->ev[l][q][0], c->ev[l][q][1]);
             c->stats.ms_kernel[l][q] = ms;
+            c->prof_sum[l][q] += ms;
+            if (c->cfg.profile && c->ev_used[l][q]) c->prof_cnt[l][q] += 1;
             c->ev_used[l][q] = false;
         }
     (void)cudaGetLastError();
@@ -352,6 +369,8 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     S.launches = c->launches;
     S.h2d_bytes = c->h2d;
     S.d2h_bytes = c->d2h;
+    c->launches_total += c->launches;
+    c->calls_total += 1;
     prof_collect(c);
     return SS_OK;
 }
@@ -405,6 +424,8 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     S.launches = c->launches;
     S.h2d_bytes = c->h2d;
     S.d2h_bytes = c->d2h;
+    c->launches_total += c->launches;
+    c->calls_total += 1;
     prof_collect(c);
     return SS_OK;
 }
@@ -532,11 +553,26 @@ ss_status ss_set_config(ss_context* c, const ss_config* cfg) {
         return fail(c, SS_ERR_INVALID_ARGUMENT, "sample_size must be 0 or a power of two in [b, 16384]");
     if (!pow2(cfg->base_case) || cfg->base_case < 256 || cfg->base_case > 16384)
         return fail(c, SS_ERR_INVALID_ARGUMENT, "base_case must be a power of two in [256, 16384]");
-    if (cfg->profile != 0 && cfg->profile != 1)
-        return fail(c, SS_ERR_INVALID_ARGUMENT, "profile must be 0 or 1");
+    if (cfg->profile < 0 || cfg->profile > 2)
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "profile must be 0, 1 or 2");
     if (cfg->ctas_per_sm < 1 || cfg->ctas_per_sm > 16)
         return fail(c, SS_ERR_INVALID_ARGUMENT, "ctas_per_sm must be in [1, 16]");
     c->cfg = *cfg;
+    return SS_OK;
+}
+
+ss_status ss_profile_totals(ss_context* c, double* ms_sum, int64_t* count, int64_t* launches,
+                            int64_t* calls, int32_t reset) {
+    if (!c) return SS_ERR_INVALID_ARGUMENT;
+    for (int l = 0; l < SS_MAX_LEVELS; ++l)
+        for (int q = 0; q < 3; ++q) {
+            if (ms_sum) ms_sum[l * 3 + q] = c->prof_sum[l][q];
+            if (count) count[l * 3 + q] = c->prof_cnt[l][q];
+            if (reset) { c->prof_sum[l][q] = 0; c->prof_cnt[l][q] = 0; }
+        }
+    if (launches) *launches = c->launches_total;
+    if (calls) *calls = c->calls_total;
+    if (reset) { c->launches_total = 0; c->calls_total = 0; }
     return SS_OK;
 }
 
