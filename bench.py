@@ -224,7 +224,7 @@ def run_ours(args, rank, world, local_rank):
         from paper_conf_ipps_ribizela19_b200 import sharded
         group_n = n * world
         k = group_n // 2
-        sel = sharded.ShardedSelect(ctx)
+        sel = sharded.ShardedSelect(sharded.CudaSteps(ctx), sharded.TorchDistComm(), b=b)
 
         def step(inp):
             return sel.select(inp, k)
