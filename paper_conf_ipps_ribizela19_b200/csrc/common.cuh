@@ -92,7 +92,7 @@ struct SelectResult {
 // last active CTA.  K2 counts per unit; K5 compacts per unit with no
 // cross-warp synchronisation.
 constexpr u32 UNIT_WARPS = 16;          // warps per CTA in K2 and K5 (512 threads)
-constexpr u64 MIN_GROUPS_PER_UNIT = 4;  // 64 elements
+constexpr u64 MIN_GROUPS_PER_UNIT = 64; // 1024 elements: small levels use few CTAs
 
 struct Chunking {
     u64 head, ngroups, tail_begin, gpw;

@@ -14,6 +14,7 @@
 #include <cstring>
 #include <new>
 #include <string>
+#include <utility>
 
 #include "kernels.cuh"
 #include "sampleselect.h"
@@ -92,6 +93,25 @@ ss_status fail(ss_context* c, ss_status s, const std::string& msg) {
 
 #define CKLAUNCH(what) CK(cudaGetLastError())
 
+// Launch with programmatic stream serialisation (PDL): the kernel may become
+// resident while its predecessor on the stream finishes; it waits for the
+// predecessor's completion inside (pdl_wait) before reading its results.
+template <typename... KArgs, typename... Args>
+cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                       Args&&... args) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = grid;
+    cfg.blockDim = block;
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
+}
+
 int log2i(int b) {
     int h = 0;
     while ((1 << h) < b) ++h;
@@ -151,8 +171,8 @@ ss_status launch_count(ss_context* c, int H, const T* in, CountArgs& a, cudaStre
 #define SS_COUNT_CASE(h)                                                     \
     case h:                                                                  \
         a.grid = count_grid<T, h>(c);                                        \
-        count_kernel<T, h><<<a.grid, K2_THREADS,                             \
-            count_smem_bytes<h, typename Traits<T>::Key>(), st>>>(in, a);    \
+        CK(launch_pdl(count_kernel<T, h>, dim3(a.grid), dim3(K2_THREADS),    \
+            count_smem_bytes<h, typename Traits<T>::Key>(), st, in, a));     \
         break;
     switch (H) {
         SS_COUNT_CASE(2) SS_COUNT_CASE(3) SS_COUNT_CASE(4) SS_COUNT_CASE(5) SS_COUNT_CASE(6)
@@ -268,8 +288,9 @@ ss_status launch_k1(ss_context* c, const T* in, int lev, int s, int b, int fixup
     K* spl = reinterpret_cast<K*>(c->d_spl) + (size_t)lev * MAX_B;
     uint8_t* eq = c->d_eq + (size_t)lev * MAX_B;
     mark(c, lev, 0, 0, st);
-    sample_tree_kernel<T><<<1, K1_THREADS, k1_smem<T>(s, B), st>>>(
-        in, c->d_ctl + lev, c->d_res, tree, spl, eq, s, b, fixup, B, c->cfg.seed, lev, final_level);
+    CK(launch_pdl(sample_tree_kernel<T>, dim3(1), dim3(K1_THREADS), k1_smem<T>(s, B), st,
+                  in, c->d_ctl + lev, c->d_res, tree, spl, eq, s, b, fixup, B, (u64)c->cfg.seed, lev,
+                  final_level));
     CKLAUNCH("sample_tree_kernel");
     mark(c, lev, 0, 1, st);
     ++c->launches;
@@ -279,7 +300,11 @@ ss_status launch_k1(ss_context* c, const T* in, int lev, int s, int b, int fixup
 template <typename T>
 ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cudaStream_t st) {
     typedef typename Traits<T>::Key K;
+    // reading R7: level 0 draws s = clamp(16 b, 4096, 16384) samples (or the
+    // configured size); deeper levels hold n_l ~ n / b elements and draw
+    // S_DEEP = max(1024, b) -- a quarter of the sort, ~1.25x the bucket size
     const int b = c->cfg.b_exact, H = log2i(b), s = sample_size(c->cfg, b);
+    const int s_deep = std::min(s, std::max(1024, b));
     const u32 B = (u32)c->cfg.base_case;
     ss_status rc;
     if ((rc = ensure_small(c))) return rc;
@@ -290,17 +315,19 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     // survivor ping-pong buffers: a level's survivors never exceed its input
     for (int i = 0; i < 2; ++i)
         if ((rc = grow(c, &c->d_buf[i], &c->cap_buf[i], n * sizeof(T)))) return rc;
-    init_kernel<<<1, 1024, 0, st>>>(c->d_ctl, SS_MAX_LEVELS + 1, c->d_totals, SS_MAX_LEVELS * MAX_B, c->d_res,
-                                    n, k);
+    int L = expected_levels(n, b, B);
+    // totals of every level are zeroed here; levels beyond the plan (the
+    // rare "incomplete" fallback) are zeroed before they run
+    CK(launch_pdl(init_kernel, dim3(1), dim3(1024), 0, st, c->d_ctl, (int)(SS_MAX_LEVELS + 1), c->d_totals,
+                  (int)((L + 1) * MAX_B), c->d_res, n, k));
     CKLAUNCH("init_kernel");
     ++c->launches;
     const u32 grid = grid_for<T>(c, H);
-    int L = expected_levels(n, b, B);
     int lev = 0;
     const T* in = d;
     for (;;) {
         for (; lev < L; ++lev) {
-            if ((rc = launch_k1<T>(c, in, lev, s, b, 1, B, 0, st))) return rc;
+            if ((rc = launch_k1<T>(c, in, lev, lev ? s_deep : s, b, 1, B, 0, st))) return rc;
             CountArgs a{};
             a.ctl = c->d_ctl + lev;
             a.ctl_next = c->d_ctl + lev + 1;
@@ -330,13 +357,13 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             f.b_count = (u32)b;
             f.grid = grid;
             mark(c, lev, 2, 0, st);
-            filter_kernel<T><<<grid, K5_THREADS, FILTER_SMEM, st>>>(in, out, f);
+            CK(launch_pdl(filter_kernel<T>, dim3(grid), dim3(K5_THREADS), FILTER_SMEM, st, in, out, f));
             CKLAUNCH("filter_kernel");
             mark(c, lev, 2, 1, st);
             ++c->launches;
             in = out;
         }
-        if ((rc = launch_k1<T>(c, in, lev, s, b, 1, B, 1, st))) return rc;
+        if ((rc = launch_k1<T>(c, in, lev, lev ? s_deep : s, b, 1, B, 1, st))) return rc;
         CK(cudaMemcpyAsync(c->h_res, c->d_res, sizeof(SelectResult), cudaMemcpyDeviceToHost, st));
         c->d2h += sizeof(SelectResult);
         CK(cudaStreamSynchronize(st));
@@ -345,6 +372,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             return fail(c, SS_ERR_INTERNAL, "recursion did not terminate");
         CK(cudaMemsetAsync(&c->d_res->incomplete, 0, sizeof(int), st));
         L = lev + 1;
+        CK(cudaMemsetAsync(c->d_totals + (size_t)lev * MAX_B, 0, sizeof(u64) * MAX_B, st));
     }
     const SelectResult& r = *c->h_res;
     std::memcpy(h_result, &r.bits, sizeof(T));
@@ -387,7 +415,7 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     if (c->cfg.profile && (rc = prof_init(c))) return rc;
     c->launches = 0;
     c->d2h = 0;
-    init_kernel<<<1, 1024, 0, st>>>(c->d_ctl, 2, c->d_totals, MAX_B, c->d_res, n, k);
+    CK(launch_pdl(init_kernel, dim3(1), dim3(1024), 0, st, c->d_ctl, 2, c->d_totals, (int)MAX_B, c->d_res, n, k));
     CKLAUNCH("init_kernel");
     ++c->launches;
     if ((rc = launch_k1<T>(c, d, 0, s, b, 0, 0, 0, st))) return rc;
