@@ -63,7 +63,8 @@ typedef struct {
     int32_t ctas_per_sm;  /* count/filter grid = ctas_per_sm * #SMs. default 4 */
     int32_t profile;      /* 1: record CUDA events around every kernel on the call's
                              stream and report per-kernel device times in ss_stats;
-                             2: only around the dominant kernel (level-0 count) */
+                             2: only around the dominant kernel (level-0 count);
+                             3: in-kernel timeline stamps (ss_stats.tl_us) */
     uint64_t seed;        /* sampling seed (reading R7). default 0x5A17 */
 } ss_config;
 
@@ -78,7 +79,12 @@ typedef struct {
     int64_t h2d_bytes;                 /* host->device bytes this call copied (host-input calls) */
     int64_t d2h_bytes;                 /* device->host bytes this call copied (result block) */
     float ms_kernel[SS_MAX_LEVELS][3]; /* profile=1: device ms of K1 (sample/tree or base
-                                          case), K2 (count+tail), K5 (filter) per level */
+                                          case), K2 (count+tail), K5 (filter) per level;
+                                          profile=3: last-CTA exit - first-CTA start */
+    float tl_us[SS_MAX_LEVELS][3][2];  /* profile=3 (timeline): [start, end] of each kernel in
+                                          us after the call's init kernel, from %globaltimer
+                                          stamps taken inside the kernels (no events, so the
+                                          PDL overlap of the chain is kept); -1 = not run */
 } ss_stats;
 
 /* ---- context --------------------------------------------------------- */

@@ -101,7 +101,8 @@ class Context:
                 "n_level": list(s.n_level[:L + 1]), "bucket": list(s.bucket[:L]),
                 "bytes_algorithmic": s.bytes_algorithmic, "launches": s.launches,
                 "h2d_bytes": s.h2d_bytes, "d2h_bytes": s.d2h_bytes,
-                "ms_kernel": [list(s.ms_kernel[l]) for l in range(L + 1)]}
+                "ms_kernel": [list(s.ms_kernel[l]) for l in range(L + 1)],
+                "tl_us": [[list(s.tl_us[l][q]) for q in range(3)] for l in range(L + 1)]}
 
     def profile_totals(self, reset: bool = False) -> dict:
         """Per-(level, kernel) device ms summed over calls made with

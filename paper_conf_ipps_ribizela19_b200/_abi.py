@@ -40,7 +40,8 @@ class SSStats(ctypes.Structure):
                 ("bytes_algorithmic", ctypes.c_double),
                 ("launches", ctypes.c_int32),
                 ("h2d_bytes", ctypes.c_int64), ("d2h_bytes", ctypes.c_int64),
-                ("ms_kernel", (ctypes.c_float * 3) * SS_MAX_LEVELS)]
+                ("ms_kernel", (ctypes.c_float * 3) * SS_MAX_LEVELS),
+                ("tl_us", ((ctypes.c_float * 2) * 3) * SS_MAX_LEVELS)]
 
 
 class SSError(RuntimeError):

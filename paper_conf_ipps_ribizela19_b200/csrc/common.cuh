@@ -79,6 +79,33 @@ struct SelectResult {
     long long n_level[32];
     int bucket[32];
     long long split_index;    // approximate: 1-based splitter index returned
+    int tl_on;                // timeline mode (profile = 3): kernels stamp tl[]
+    int pad_;
+    u64 t_init;               // %globaltimer at the init kernel (timeline origin)
+    // timeline: per (level, kernel) slot, [0] = ~(earliest CTA start after
+    // pdl_wait) and [1] = latest CTA exit, %globaltimer ns (atomicMax both)
+    u64 tl[32 * 3][2];
+};
+
+__device__ __forceinline__ u64 gtimer() {
+    u64 t;
+    asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+    return t;
+}
+
+// Scope guard stamping a kernel's device-side interval into the timeline
+// (one atomic per CTA on entry and exit; inert unless res->tl_on).
+struct TimelineScope {
+    u64* slot;
+    __device__ __forceinline__ TimelineScope(SelectResult* r, int level, int kernel) : slot(nullptr) {
+        if (r && level < 32 && r->tl_on) {
+            slot = r->tl[level * 3 + kernel];
+            if (threadIdx.x == 0) atomicMax(reinterpret_cast<unsigned long long*>(slot), ~gtimer());
+        }
+    }
+    __device__ __forceinline__ ~TimelineScope() {
+        if (slot && threadIdx.x == 0) atomicMax(reinterpret_cast<unsigned long long*>(slot + 1), gtimer());
+    }
 };
 
 // ------------------------------------------------------------ chunking ----
@@ -92,7 +119,7 @@ struct SelectResult {
 // last active CTA.  K2 counts per unit; K5 compacts per unit with no
 // cross-warp synchronisation.
 constexpr u32 UNIT_WARPS = 16;          // warps per CTA in K2 and K5 (512 threads)
-constexpr u64 MIN_GROUPS_PER_UNIT = 64; // 1024 elements: small levels use few CTAs
+constexpr u64 MIN_GROUPS_PER_UNIT = 4;  // 64 elements: small levels still spread over many warps
 
 struct Chunking {
     u64 head, ngroups, tail_begin, gpw;

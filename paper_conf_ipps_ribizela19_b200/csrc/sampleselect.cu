@@ -42,6 +42,8 @@ struct ss_context {
     u64* d_tree = nullptr;       // [SS_MAX_LEVELS][MAX_B] keys (u32 keys use the same bytes)
     u64* d_spl = nullptr;
     uint8_t* d_eq = nullptr;     // [SS_MAX_LEVELS][MAX_B]
+    u64* d_sorted = nullptr;     // [SS_MAX_LEVELS][MAX_S] sorted sample keys (wide K1)
+    u64* d_sample0 = nullptr;    // [MAX_S] level-0 sample keys (gathered by the init kernel)
     SelectResult* h_res = nullptr;
     // record of the last ss_step_count (per-CTA counts feed ss_step_filter)
     const void* step_ptr = nullptr;
@@ -62,6 +64,10 @@ struct ss_context {
 };
 
 static constexpr u32 MAX_GRID = 2048;
+static constexpr int MAX_S = 16384;
+// sample sizes up to this are ranked by the wide K1 (s/32 CTAs, s^2 pairs);
+// larger samples (approximate b = 1024) use the one-CTA bitonic K1
+static constexpr int WIDE_K1_MAX_S = 4096;
 
 namespace {
 
@@ -213,6 +219,8 @@ ss_status set_k1_attrs(ss_context* c) {
     CK(cudaFuncSetAttribute(tree_from_keys_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                             (int)(16384 * sizeof(K))));
     CK(cudaFuncSetAttribute(filter_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)FILTER_SMEM));
+    CK(cudaFuncSetAttribute(sample_rank_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)(16384 * sizeof(K))));
     // one carveout (all shared) for every kernel of the path: no L1/shared
     // reconfiguration between consecutive kernels
 #ifdef SS_CARVEOUT
@@ -233,6 +241,8 @@ ss_status ensure_small(ss_context* c) {
     CK(cudaMalloc(&c->d_tree, sizeof(u64) * SS_MAX_LEVELS * MAX_B));
     CK(cudaMalloc(&c->d_spl, sizeof(u64) * SS_MAX_LEVELS * MAX_B));
     CK(cudaMalloc(&c->d_eq, (size_t)SS_MAX_LEVELS * MAX_B));
+    CK(cudaMalloc(&c->d_sorted, sizeof(u64) * SS_MAX_LEVELS * MAX_S));
+    CK(cudaMalloc(&c->d_sample0, sizeof(u64) * MAX_S));
     CK(cudaMallocHost(&c->h_res, sizeof(SelectResult)));
     return SS_OK;
 }
@@ -248,13 +258,35 @@ ss_status prof_init(ss_context* c) {
 
 // Record the start (e=0) / end (e=1) event of kernel q at level l.
 inline void mark(ss_context* c, int l, int q, int e, cudaStream_t st) {
-    if (!c->cfg.profile || l >= SS_MAX_LEVELS) return;
+    if (!c->cfg.profile || c->cfg.profile == 3 || l >= SS_MAX_LEVELS) return;
     if (c->cfg.profile == 2 && !(l == 0 && q == 1)) return;   // dominant kernel only
     cudaEventRecord(c->ev[l][q][e], st);
     if (e) c->ev_used[l][q] = true;
 }
 
+// bytes of the result block read back per call (the timeline only in profile=3)
+size_t res_bytes(const ss_context* c) {
+    return c->cfg.profile == 3 ? sizeof(SelectResult) : offsetof(SelectResult, tl_on);
+}
+
 void prof_collect(ss_context* c) {
+    if (c->cfg.profile == 3) {
+        const SelectResult& r = *c->h_res;
+        for (int l = 0; l < SS_MAX_LEVELS; ++l)
+            for (int q = 0; q < 3; ++q) {
+                const u64 a = ~r.tl[l * 3 + q][0], b = r.tl[l * 3 + q][1];
+                const bool ran = r.tl[l * 3 + q][0] != 0 && b != 0;
+                c->stats.tl_us[l][q][0] = ran ? (float)((double)(long long)(a - r.t_init) * 1e-3) : -1.f;
+                c->stats.tl_us[l][q][1] = ran ? (float)((double)(long long)(b - r.t_init) * 1e-3) : -1.f;
+                const float ms = ran ? (float)((double)(long long)(b - a) * 1e-6) : 0.f;
+                c->stats.ms_kernel[l][q] = ms;
+                if (ran) {
+                    c->prof_sum[l][q] += ms;
+                    c->prof_cnt[l][q] += 1;
+                }
+            }
+        return;
+    }
     for (int l = 0; l < SS_MAX_LEVELS; ++l)
         for (int q = 0; q < 3; ++q) {
             float ms = 0.f;
@@ -297,6 +329,23 @@ ss_status launch_k1(ss_context* c, const T* in, int lev, int s, int b, int fixup
     return SS_OK;
 }
 
+// Wide K1: gather + rank the level's sample on s/32 CTAs (or the base case).
+template <typename T>
+ss_status launch_k1_wide(ss_context* c, const T* in, int lev, int s, u32 B, cudaStream_t st,
+                         const void* presampled = nullptr) {
+    typedef typename Traits<T>::Key K;
+    K* sorted = reinterpret_cast<K*>(c->d_sorted) + (size_t)lev * MAX_S;
+    mark(c, lev, 0, 0, st);
+    CK(launch_pdl(sample_rank_kernel<T>, dim3((u32)s / 32u), dim3(K1R_THREADS),
+                  (size_t)std::max<u32>((u32)s, B) * sizeof(K), st,
+                  in, c->d_ctl + lev, c->d_res, sorted, s, B, (u64)c->cfg.seed, lev,
+                  reinterpret_cast<const K*>(presampled)));
+    CKLAUNCH("sample_rank_kernel");
+    mark(c, lev, 0, 1, st);
+    ++c->launches;
+    return SS_OK;
+}
+
 template <typename T>
 ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cudaStream_t st) {
     typedef typename Traits<T>::Key K;
@@ -318,8 +367,12 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     int L = expected_levels(n, b, B);
     // totals of every level are zeroed here; levels beyond the plan (the
     // rare "incomplete" fallback) are zeroed before they run
-    CK(launch_pdl(init_kernel, dim3(1), dim3(1024), 0, st, c->d_ctl, (int)(SS_MAX_LEVELS + 1), c->d_totals,
-                  (int)((L + 1) * MAX_B), c->d_res, n, k));
+    // level 0's sample is gathered by the init kernel when the wide K1 ranks it
+    const bool pre0 = L > 0 && s <= WIDE_K1_MAX_S;
+    K* sample0 = pre0 ? reinterpret_cast<K*>(c->d_sample0) : nullptr;
+    CK(launch_pdl(init_kernel<T>, dim3(pre0 ? (u32)s / 256u : 1u), dim3(256), 0, st, c->d_ctl,
+                  (int)(SS_MAX_LEVELS + 1), c->d_totals, (int)((L + 1) * MAX_B), c->d_res, n, k,
+                  (int)(c->cfg.profile == 3), d, s, (u64)c->cfg.seed, sample0));
     CKLAUNCH("init_kernel");
     ++c->launches;
     const u32 grid = grid_for<T>(c, H);
@@ -327,8 +380,19 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     const T* in = d;
     for (;;) {
         for (; lev < L; ++lev) {
-            if ((rc = launch_k1<T>(c, in, lev, lev ? s_deep : s, b, 1, B, 0, st))) return rc;
+            const int sl = lev ? s_deep : s;
+            const bool wide = sl <= WIDE_K1_MAX_S;
+            if (wide) {
+                if ((rc = launch_k1_wide<T>(c, in, lev, sl, B, st, lev == 0 ? sample0 : nullptr))) return rc;
+            } else if ((rc = launch_k1<T>(c, in, lev, sl, b, 1, B, 0, st))) {
+                return rc;
+            }
             CountArgs a{};
+            if (wide) {
+                a.sorted = reinterpret_cast<K*>(c->d_sorted) + (size_t)lev * MAX_S;
+                a.s = sl;
+                a.fixup = 1;
+            }
             a.ctl = c->d_ctl + lev;
             a.ctl_next = c->d_ctl + lev + 1;
             a.res = c->d_res;
@@ -356,6 +420,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             f.warp_counts = c->d_warp_counts;
             f.b_count = (u32)b;
             f.grid = grid;
+            f.level = lev;
             mark(c, lev, 2, 0, st);
             CK(launch_pdl(filter_kernel<T>, dim3(grid), dim3(K5_THREADS), FILTER_SMEM, st, in, out, f));
             CKLAUNCH("filter_kernel");
@@ -364,8 +429,8 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             in = out;
         }
         if ((rc = launch_k1<T>(c, in, lev, lev ? s_deep : s, b, 1, B, 1, st))) return rc;
-        CK(cudaMemcpyAsync(c->h_res, c->d_res, sizeof(SelectResult), cudaMemcpyDeviceToHost, st));
-        c->d2h += sizeof(SelectResult);
+        CK(cudaMemcpyAsync(c->h_res, c->d_res, res_bytes(c), cudaMemcpyDeviceToHost, st));
+        c->d2h += res_bytes(c);
         CK(cudaStreamSynchronize(st));
         if (c->h_res->done) break;
         if (!c->h_res->incomplete || lev >= SS_MAX_LEVELS - 2)
@@ -415,11 +480,23 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     if (c->cfg.profile && (rc = prof_init(c))) return rc;
     c->launches = 0;
     c->d2h = 0;
-    CK(launch_pdl(init_kernel, dim3(1), dim3(1024), 0, st, c->d_ctl, 2, c->d_totals, (int)MAX_B, c->d_res, n, k));
+    const bool wide = s <= WIDE_K1_MAX_S;
+    K* sample0 = wide ? reinterpret_cast<K*>(c->d_sample0) : nullptr;
+    CK(launch_pdl(init_kernel<T>, dim3(wide ? (u32)s / 256u : 1u), dim3(256), 0, st, c->d_ctl, 2, c->d_totals,
+                  (int)MAX_B, c->d_res, n, k, (int)(c->cfg.profile == 3), d, s, (u64)c->cfg.seed, sample0));
     CKLAUNCH("init_kernel");
     ++c->launches;
-    if ((rc = launch_k1<T>(c, d, 0, s, b, 0, 0, 0, st))) return rc;
+    if (wide) {
+        if ((rc = launch_k1_wide<T>(c, d, 0, s, 0, st, sample0))) return rc;
+    } else if ((rc = launch_k1<T>(c, d, 0, s, b, 0, 0, 0, st))) {
+        return rc;
+    }
     CountArgs a{};
+    if (wide) {
+        a.sorted = reinterpret_cast<K*>(c->d_sorted);
+        a.s = s;
+        a.fixup = 0;
+    }
     a.ctl = c->d_ctl;
     a.ctl_next = c->d_ctl + 1;
     a.res = c->d_res;
@@ -436,8 +513,8 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     if ((rc = launch_count<T>(c, H, d, a, st))) return rc;
     mark(c, 0, 1, 1, st);
     ++c->launches;
-    CK(cudaMemcpyAsync(c->h_res, c->d_res, sizeof(SelectResult), cudaMemcpyDeviceToHost, st));
-    c->d2h += sizeof(SelectResult);
+    CK(cudaMemcpyAsync(c->h_res, c->d_res, res_bytes(c), cudaMemcpyDeviceToHost, st));
+    c->d2h += res_bytes(c);
     CK(cudaStreamSynchronize(st));
     const SelectResult& r = *c->h_res;
     if (!r.done) return fail(c, SS_ERR_INTERNAL, "approximate select produced no result");
@@ -557,6 +634,8 @@ void ss_destroy(ss_context* c) {
     cudaFree(c->d_tree);
     cudaFree(c->d_spl);
     cudaFree(c->d_eq);
+    cudaFree(c->d_sorted);
+    cudaFree(c->d_sample0);
     if (c->h_res) cudaFreeHost(c->h_res);
     if (c->ev_ready)
         for (int l = 0; l < SS_MAX_LEVELS; ++l)
@@ -581,8 +660,8 @@ ss_status ss_set_config(ss_context* c, const ss_config* cfg) {
         return fail(c, SS_ERR_INVALID_ARGUMENT, "sample_size must be 0 or a power of two in [b, 16384]");
     if (!pow2(cfg->base_case) || cfg->base_case < 256 || cfg->base_case > 16384)
         return fail(c, SS_ERR_INVALID_ARGUMENT, "base_case must be a power of two in [256, 16384]");
-    if (cfg->profile < 0 || cfg->profile > 2)
-        return fail(c, SS_ERR_INVALID_ARGUMENT, "profile must be 0, 1 or 2");
+    if (cfg->profile < 0 || cfg->profile > 3)
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "profile must be 0, 1, 2 or 3");
     if (cfg->ctas_per_sm < 1 || cfg->ctas_per_sm > 16)
         return fail(c, SS_ERR_INVALID_ARGUMENT, "ctas_per_sm must be in [1, 16]");
     c->cfg = *cfg;

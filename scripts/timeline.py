@@ -1,0 +1,44 @@
+"""Device timeline of one selection (profile=3: %globaltimer stamps inside the
+kernels, PDL overlap intact).  `python scripts/timeline.py [log2n] [b] [mode]`"""
+import os, sys, time
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np, torch
+import datagen
+import paper_conf_ipps_ribizela19_b200 as ss
+
+log2n = int(sys.argv[1]) if len(sys.argv) > 1 else 28
+b = int(sys.argv[2]) if len(sys.argv) > 2 else 256
+mode = sys.argv[3] if len(sys.argv) > 3 else "exact"
+n = 1 << log2n
+x = torch.from_numpy(datagen.uniform(n, np.float32, seed=datagen.dataset_seed(5, 0))).cuda()
+ctx = ss.Context(0)
+if mode == "exact":
+    ctx.configure(b_exact=b)
+run = (lambda: ctx.select(x, n // 2)) if mode == "exact" else (lambda: ctx.approx_select(x, n // 2, b))
+for _ in range(5):
+    run()
+torch.cuda.synchronize()
+ctx.configure(profile=3)
+R = 20
+acc = None
+for _ in range(R):
+    run()
+    st = ctx.stats()
+    tl = np.array(st["tl_us"], dtype=np.float64)
+    acc = tl if acc is None else acc + tl
+tl = acc / R
+names = ["K1", "K2", "K5"]
+print(f"n=2^{log2n} b={b} {mode}: n_level={st['n_level']}  (mean of {R} calls, us after init)")
+for l in range(tl.shape[0]):
+    for q in range(3):
+        s0, s1 = tl[l][q]
+        if s0 >= 0 and s1 > 0:
+            print(f"  L{l} {names[q]}: start {s0:8.1f}  end {s1:8.1f}  dur {s1 - s0:7.1f}")
+ctx.configure(profile=0)
+torch.cuda.synchronize()
+ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+ev0.record()
+for _ in range(R):
+    run()
+ev1.record(); torch.cuda.synchronize()
+print(f"  per call (events, profile=0): {ev0.elapsed_time(ev1) / R * 1e3:.1f} us")
