@@ -65,6 +65,9 @@ typedef struct {
                              stream and report per-kernel device times in ss_stats;
                              2: only around the dominant kernel (level-0 count);
                              3: in-kernel timeline stamps (ss_stats.tl_us) */
+    int32_t b_deep;       /* buckets of the levels after the first: 0 = b_exact, else a
+                             power of two in [4, 256] (each level is a full SampleSelect
+                             level of Fig. 1; only its bucket count differs) */
     uint64_t seed;        /* sampling seed (reading R7). default 0x5A17 */
 } ss_config;
 

@@ -30,7 +30,8 @@ EXPORTS = [
 class SSConfig(ctypes.Structure):
     _fields_ = [("b_exact", ctypes.c_int32), ("sample_size", ctypes.c_int32),
                 ("base_case", ctypes.c_int32), ("ctas_per_sm", ctypes.c_int32),
-                ("profile", ctypes.c_int32), ("seed", ctypes.c_uint64)]
+                ("profile", ctypes.c_int32), ("b_deep", ctypes.c_int32),
+                ("seed", ctypes.c_uint64)]
 
 
 class SSStats(ctypes.Structure):

@@ -79,6 +79,8 @@ struct SelectResult {
     long long n_level[32];
     int bucket[32];
     long long split_index;    // approximate: 1-based splitter index returned
+    unsigned int seq;         // host mirror only: publish sequence number, written last
+    int pad_seq;
     int tl_on;                // timeline mode (profile = 3): kernels stamp tl[]
     int pad_;
     u64 t_init;               // %globaltimer at the init kernel (timeline origin)

@@ -9,6 +9,8 @@
 // case (rare: an unlucky sample) more levels are enqueued.  One device->host
 // copy per call returns the answer; there is no per-level host round trip.
 #include <algorithm>
+#include <atomic>
+#include <cstddef>
 #include <cstdlib>
 #include <cstdio>
 #include <cstring>
@@ -44,7 +46,9 @@ struct ss_context {
     uint8_t* d_eq = nullptr;     // [SS_MAX_LEVELS][MAX_B]
     u64* d_sorted = nullptr;     // [SS_MAX_LEVELS][MAX_S] sorted sample keys (wide K1)
     u64* d_sample0 = nullptr;    // [MAX_S] level-0 sample keys (gathered by the init kernel)
-    SelectResult* h_res = nullptr;
+    SelectResult* h_res = nullptr;   // mapped pinned mirror of d_res (written by publish_kernel)
+    SelectResult* h_res_dev = nullptr;
+    u32 seq = 0;
     // record of the last ss_step_count (per-CTA counts feed ss_step_filter)
     const void* step_ptr = nullptr;
     u64 step_n = 0;
@@ -205,10 +209,11 @@ u32 grid_for(ss_context* c, int H) {
     }
 }
 
+// K1's dynamic smem holds the s sample keys (the base case keeps its keys in registers)
 template <typename T>
-size_t k1_smem(int s, u32 B) {
+size_t k1_smem(int s, u32 /*B*/) {
     typedef typename Traits<T>::Key K;
-    return (size_t)std::max<u32>((u32)s, B) * sizeof(K);
+    return (size_t)s * sizeof(K);
 }
 
 template <typename T>
@@ -243,7 +248,9 @@ ss_status ensure_small(ss_context* c) {
     CK(cudaMalloc(&c->d_eq, (size_t)SS_MAX_LEVELS * MAX_B));
     CK(cudaMalloc(&c->d_sorted, sizeof(u64) * SS_MAX_LEVELS * MAX_S));
     CK(cudaMalloc(&c->d_sample0, sizeof(u64) * MAX_S));
-    CK(cudaMallocHost(&c->h_res, sizeof(SelectResult)));
+    CK(cudaHostAlloc(&c->h_res, sizeof(SelectResult), cudaHostAllocMapped));
+    std::memset(c->h_res, 0, sizeof(SelectResult));
+    CK(cudaHostGetDevicePointer((void**)&c->h_res_dev, c->h_res, 0));
     return SS_OK;
 }
 
@@ -267,6 +274,31 @@ inline void mark(ss_context* c, int l, int q, int e, cudaStream_t st) {
 // bytes of the result block read back per call (the timeline only in profile=3)
 size_t res_bytes(const ss_context* c) {
     return c->cfg.profile == 3 ? sizeof(SelectResult) : offsetof(SelectResult, tl_on);
+}
+
+// Enqueue the result hand-off and wait for it: the publish kernel writes the
+// result block into the mapped host mirror and then the new sequence number;
+// the host spins on that word (checking the stream for errors now and then).
+ss_status publish_and_wait(ss_context* c, cudaStream_t st) {
+    const u32 seq = ++c->seq;
+    const u32 nwords = (u32)(res_bytes(c) / 4);
+    const u32 seq_word = (u32)(offsetof(SelectResult, seq) / 4);
+    CK(launch_pdl(publish_kernel, dim3(1), dim3(128), 0, st, reinterpret_cast<const u32*>(c->d_res),
+                  reinterpret_cast<u32*>(c->h_res_dev), nwords, seq_word, seq));
+    CKLAUNCH("publish_kernel");
+    ++c->launches;
+    c->d2h += res_bytes(c);
+    volatile u32* flag = &c->h_res->seq;
+    for (u64 spin = 1;; ++spin) {
+        if (*flag == seq) break;
+        if ((spin & 1023) == 0) {
+            const cudaError_t e = cudaStreamQuery(st);
+            if (e != cudaSuccess && e != cudaErrorNotReady) CK(e);
+            if (e == cudaSuccess && *flag != seq) return fail(c, SS_ERR_INTERNAL, "result hand-off lost");
+        }
+    }
+    std::atomic_thread_fence(std::memory_order_acquire);
+    return SS_OK;
 }
 
 void prof_collect(ss_context* c) {
@@ -300,13 +332,13 @@ void prof_collect(ss_context* c) {
     (void)cudaGetLastError();
 }
 
-int expected_levels(u64 n, int b, u32 B) {
-    // n_{l+1} ~ n_l / b times the size bias of the bucket holding k (~1.1 for
-    // s/b = 16); plan with 1.5x slack, fall back to more levels if needed.
+int expected_levels(u64 n, int b0, int bd, u32 B) {
+    // n_{l+1} ~ n_l / b_l times the size bias of the bucket holding k (~1.1
+    // for s/b = 16); plan with 1.5x slack, fall back to more levels if needed.
     int L = 0;
     double m = (double)n;
     while (m > (double)B && L < SS_MAX_LEVELS - 2) {
-        m = m * 1.5 / b;
+        m = m * 1.5 / (L ? bd : b0);
         ++L;
     }
     return L;
@@ -337,7 +369,7 @@ ss_status launch_k1_wide(ss_context* c, const T* in, int lev, int s, u32 B, cuda
     K* sorted = reinterpret_cast<K*>(c->d_sorted) + (size_t)lev * MAX_S;
     mark(c, lev, 0, 0, st);
     CK(launch_pdl(sample_rank_kernel<T>, dim3((u32)s / 32u), dim3(K1R_THREADS),
-                  (size_t)std::max<u32>((u32)s, B) * sizeof(K), st,
+                  k1_smem<T>(s, B), st,
                   in, c->d_ctl + lev, c->d_res, sorted, s, B, (u64)c->cfg.seed, lev,
                   reinterpret_cast<const K*>(presampled)));
     CKLAUNCH("sample_rank_kernel");
@@ -352,8 +384,10 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     // reading R7: level 0 draws s = clamp(16 b, 4096, 16384) samples (or the
     // configured size); deeper levels hold n_l ~ n / b elements and draw
     // S_DEEP = max(1024, b) -- a quarter of the sort, ~1.25x the bucket size
-    const int b = c->cfg.b_exact, H = log2i(b), s = sample_size(c->cfg, b);
-    const int s_deep = std::min(s, std::max(1024, b));
+    // level 0 uses b_exact buckets, deeper levels b_deep (default: the same)
+    const int b0 = c->cfg.b_exact, bd = c->cfg.b_deep ? c->cfg.b_deep : b0;
+    const int s = sample_size(c->cfg, b0);
+    const int s_deep = std::min(sample_size(c->cfg, bd), std::max(1024, bd));
     const u32 B = (u32)c->cfg.base_case;
     ss_status rc;
     if ((rc = ensure_small(c))) return rc;
@@ -364,7 +398,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     // survivor ping-pong buffers: a level's survivors never exceed its input
     for (int i = 0; i < 2; ++i)
         if ((rc = grow(c, &c->d_buf[i], &c->cap_buf[i], n * sizeof(T)))) return rc;
-    int L = expected_levels(n, b, B);
+    int L = expected_levels(n, b0, bd, B);
     // totals of every level are zeroed here; levels beyond the plan (the
     // rare "incomplete" fallback) are zeroed before they run
     // level 0's sample is gathered by the init kernel when the wide K1 ranks it
@@ -375,11 +409,12 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
                   (int)(c->cfg.profile == 3), d, s, (u64)c->cfg.seed, sample0));
     CKLAUNCH("init_kernel");
     ++c->launches;
-    const u32 grid = grid_for<T>(c, H);
     int lev = 0;
     const T* in = d;
     for (;;) {
         for (; lev < L; ++lev) {
+            const int b = lev ? bd : b0, H = log2i(b);
+            const u32 grid = grid_for<T>(c, H);
             const int sl = lev ? s_deep : s;
             const bool wide = sl <= WIDE_K1_MAX_S;
             if (wide) {
@@ -428,10 +463,8 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             ++c->launches;
             in = out;
         }
-        if ((rc = launch_k1<T>(c, in, lev, lev ? s_deep : s, b, 1, B, 1, st))) return rc;
-        CK(cudaMemcpyAsync(c->h_res, c->d_res, res_bytes(c), cudaMemcpyDeviceToHost, st));
-        c->d2h += res_bytes(c);
-        CK(cudaStreamSynchronize(st));
+        if ((rc = launch_k1<T>(c, in, lev, lev ? s_deep : s, lev ? bd : b0, 1, B, 1, st))) return rc;
+        if ((rc = publish_and_wait(c, st))) return rc;
         if (c->h_res->done) break;
         if (!c->h_res->incomplete || lev >= SS_MAX_LEVELS - 2)
             return fail(c, SS_ERR_INTERNAL, "recursion did not terminate");
@@ -513,9 +546,7 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     if ((rc = launch_count<T>(c, H, d, a, st))) return rc;
     mark(c, 0, 1, 1, st);
     ++c->launches;
-    CK(cudaMemcpyAsync(c->h_res, c->d_res, res_bytes(c), cudaMemcpyDeviceToHost, st));
-    c->d2h += res_bytes(c);
-    CK(cudaStreamSynchronize(st));
+    if ((rc = publish_and_wait(c, st))) return rc;
     const SelectResult& r = *c->h_res;
     if (!r.done) return fail(c, SS_ERR_INTERNAL, "approximate select produced no result");
     std::memcpy(h_result, &r.bits, sizeof(T));
@@ -594,6 +625,7 @@ ss_status ss_create(int device, ss_context** out) {
     if (!c) return SS_ERR_OUT_OF_MEMORY;
     c->device = device;
     c->cfg.b_exact = 256;
+    c->cfg.b_deep = 0;
     c->cfg.sample_size = 0;
     c->cfg.base_case = 16384;
     c->cfg.ctas_per_sm = 4;
@@ -655,8 +687,10 @@ ss_status ss_set_config(ss_context* c, const ss_config* cfg) {
     if (!c || !cfg) return SS_ERR_INVALID_ARGUMENT;
     if (!pow2(cfg->b_exact) || cfg->b_exact < 4 || cfg->b_exact > 256)
         return fail(c, SS_ERR_INVALID_ARGUMENT, "b_exact must be a power of two in [4, 256]");
+    if (cfg->b_deep != 0 && (!pow2(cfg->b_deep) || cfg->b_deep < 4 || cfg->b_deep > 256))
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "b_deep must be 0 or a power of two in [4, 256]");
     if (cfg->sample_size != 0 && (!pow2(cfg->sample_size) || cfg->sample_size > 16384 ||
-                                  cfg->sample_size < cfg->b_exact))
+                                  cfg->sample_size < std::max(cfg->b_exact, cfg->b_deep)))
         return fail(c, SS_ERR_INVALID_ARGUMENT, "sample_size must be 0 or a power of two in [b, 16384]");
     if (!pow2(cfg->base_case) || cfg->base_case < 256 || cfg->base_case > 16384)
         return fail(c, SS_ERR_INVALID_ARGUMENT, "base_case must be a power of two in [256, 16384]");

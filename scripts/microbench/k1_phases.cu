@@ -15,8 +15,9 @@ __global__ void __launch_bounds__(1024) probe(const u32* __restrict__ src, u32 s
     extern __shared__ __align__(16) unsigned char smem_raw[];
     u32* keys = reinterpret_cast<u32*>(smem_raw);
     __shared__ u32 spl_s[MAX_B];
-    __shared__ u32 hist[256];
-    __shared__ u32 misc[4];
+    __shared__ u32 hist[32 * 256];
+    __shared__ u32 misc[16];
+    __shared__ u32 red[64];
     __syncthreads();
     long long t0 = clock64();
     u32 acc = 0;
@@ -33,9 +34,7 @@ __global__ void __launch_bounds__(1024) probe(const u32* __restrict__ src, u32 s
             block_build_tree<u32>(keys, s, 256, 1, spl_s, out, out + 1024, (uint8_t*)(out + 2048));
             __syncthreads();
         } else if (MODE == 3) {   // base case radix select of s keys
-            for (u32 i = threadIdx.x; i < s; i += blockDim.x) keys[i] = load_key(data + i + r);
-            __syncthreads();
-            u32 v = block_radix_select<u32>(keys, s, s / 2, hist, misc);
+            u32 v = block_radix_select<float>(data + r, s, s / 2, hist, misc, red);
             acc += v;
             __syncthreads();
         }
@@ -83,6 +82,10 @@ int main() {
         run<2>("gather+sort+tree (2^28)", s, src, data, n, cyc, out);
         run<2>("gather+sort+tree (2^20)", s, src, data, 1u << 20, cyc, out);
     }
-    for (u32 s : {1024u, 3712u, 16384u}) run<3>("base radix select", s, src, data, n, cyc, out);
+    for (u32 s : {1024u, 3712u, 16384u}) run<3>("base radix select (U[0,1))", s, src, data, n, cyc, out);
+    // narrow range: values 0.5 + [0, 1e-4)
+    for (auto& x : h) x = 0.5f + 1e-4f * U(rng);
+    CK(cudaMemcpy(data, h.data(), h.size() * 4, cudaMemcpyHostToDevice));
+    for (u32 s : {1024u, 3712u, 15000u, 16384u}) run<3>("base radix select (narrow)", s, src, data, n, cyc, out);
     return 0;
 }

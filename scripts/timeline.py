@@ -9,11 +9,12 @@ import paper_conf_ipps_ribizela19_b200 as ss
 log2n = int(sys.argv[1]) if len(sys.argv) > 1 else 28
 b = int(sys.argv[2]) if len(sys.argv) > 2 else 256
 mode = sys.argv[3] if len(sys.argv) > 3 else "exact"
+bd = int(sys.argv[4]) if len(sys.argv) > 4 else 0
 n = 1 << log2n
 x = torch.from_numpy(datagen.uniform(n, np.float32, seed=datagen.dataset_seed(5, 0))).cuda()
 ctx = ss.Context(0)
 if mode == "exact":
-    ctx.configure(b_exact=b)
+    ctx.configure(b_exact=b, b_deep=bd)
 run = (lambda: ctx.select(x, n // 2)) if mode == "exact" else (lambda: ctx.approx_select(x, n // 2, b))
 for _ in range(5):
     run()
@@ -28,7 +29,7 @@ for _ in range(R):
     acc = tl if acc is None else acc + tl
 tl = acc / R
 names = ["K1", "K2", "K5"]
-print(f"n=2^{log2n} b={b} {mode}: n_level={st['n_level']}  (mean of {R} calls, us after init)")
+print(f"n=2^{log2n} b={b} b_deep={bd} {mode}: n_level={st['n_level']}  (mean of {R} calls, us after init)")
 for l in range(tl.shape[0]):
     for q in range(3):
         s0, s1 = tl[l][q]
