@@ -104,6 +104,12 @@ class Context:
                 "ms_kernel": [list(s.ms_kernel[l]) for l in range(L + 1)],
                 "tl_us": [[list(s.tl_us[l][q]) for q in range(3)] for l in range(L + 1)]}
 
+    def raw_tl(self):
+        """profile=3: the full 32x3 timeline (us after init; -1 = not stamped)."""
+        s = SSStats()
+        self._check(self._lib.ss_last_stats(self._h, ctypes.byref(s)))
+        return [[list(s.tl_us[l][q]) for q in range(3)] for l in range(_abi.SS_MAX_LEVELS)]
+
     def profile_totals(self, reset: bool = False) -> dict:
         """Per-(level, kernel) device ms summed over calls made with
         profile=1, launch and call counts since the last reset."""

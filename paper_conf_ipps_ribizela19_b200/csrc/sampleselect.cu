@@ -17,6 +17,8 @@
 #include <new>
 #include <string>
 #include <utility>
+#include <vector>
+#include <type_traits>
 
 #include "kernels.cuh"
 #include "sampleselect.h"
@@ -40,7 +42,6 @@ struct ss_context {
     u64* d_totals = nullptr;     // [SS_MAX_LEVELS][MAX_B]
     u32* d_cta_counts = nullptr; // [MAX_GRID][MAX_B]
     u32* d_warp_counts = nullptr; // [MAX_GRID][UNIT_WARPS][256]
-    u64* d_offsets = nullptr;    // [MAX_GRID]
     u64* d_tree = nullptr;       // [SS_MAX_LEVELS][MAX_B] keys (u32 keys use the same bytes)
     u64* d_spl = nullptr;
     uint8_t* d_eq = nullptr;     // [SS_MAX_LEVELS][MAX_B]
@@ -48,7 +49,31 @@ struct ss_context {
     u64* d_sample0 = nullptr;    // [MAX_S] level-0 sample keys (gathered by the init kernel)
     SelectResult* h_res = nullptr;   // mapped pinned mirror of d_res (written by publish_kernel)
     SelectResult* h_res_dev = nullptr;
-    u32 seq = 0;
+    u32 seq = 0;                     // publishes issued (host count, lockstep with *d_seq)
+    u32* d_seq = nullptr;            // device publish counter
+    // CUDA graphs of whole calls (init + levels + final K1 + publish), one per
+    // (dtype, input, n, plan); the rank k is patched into the init node
+    struct GraphEntry {
+        bool used = false;
+        int dt = -1;
+        const void* ptr = nullptr;
+        u64 n = 0;
+        int b0 = 0, bd = 0, s = 0, sd = 0, L = 0, prof = 0;
+        u32 B = 0;
+        u64 seed = 0;
+        cudaGraph_t graph = nullptr;       // kept: the init node handle belongs to it
+        cudaGraphExec_t exec = nullptr;
+        cudaGraphNode_t init_node = nullptr;
+        cudaKernelNodeParams init_params{};
+        void* init_args[16] = {};
+        unsigned char init_store[256] = {};   // backing store of the init kernel's arguments
+        size_t k_offset = 0;                  // where k lives in init_store
+        int kernels = 0;
+        u64 stamp = 0;
+    } graphs[8];
+    u64 graph_clock = 0;
+    cudaStream_t cap_st = nullptr;   // capture stream (graphs are captured off the caller's stream)
+    bool use_graphs = true;
     // record of the last ss_step_count (per-CTA counts feed ss_step_filter)
     const void* step_ptr = nullptr;
     u64 step_n = 0;
@@ -122,6 +147,10 @@ cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t s
     return cudaLaunchKernelEx(&cfg, kernel, std::forward<Args>(args)...);
 }
 
+template <typename T> constexpr int dt_code() {
+    return std::is_same<T, float>::value ? 1 : std::is_same<T, double>::value ? 2 : std::is_same<T, int>::value ? 3 : 4;
+}
+
 int log2i(int b) {
     int h = 0;
     while ((1 << h) < b) ++h;
@@ -148,6 +177,11 @@ ss_status grow(ss_context* c, void** p, size_t* cap, size_t need) {
         cudaFree(*p);
         *p = nullptr;
         *cap = 0;
+    }
+    for (auto& e : c->graphs) {   // captured graphs hold the old buffer addresses
+        if (e.exec) cudaGraphExecDestroy(e.exec);
+        if (e.graph) cudaGraphDestroy(e.graph);
+        e = ss_context::GraphEntry();
     }
     size_t alloc = need + need / 16 + 256;
     CK(cudaMalloc(p, alloc));
@@ -242,7 +276,6 @@ ss_status ensure_small(ss_context* c) {
     CK(cudaMalloc(&c->d_totals, sizeof(u64) * SS_MAX_LEVELS * MAX_B));
     CK(cudaMalloc(&c->d_cta_counts, sizeof(u32) * (size_t)MAX_GRID * MAX_B));
     CK(cudaMalloc(&c->d_warp_counts, sizeof(u32) * (size_t)MAX_GRID * UNIT_WARPS * 256));
-    CK(cudaMalloc(&c->d_offsets, sizeof(u64) * MAX_GRID));
     CK(cudaMalloc(&c->d_tree, sizeof(u64) * SS_MAX_LEVELS * MAX_B));
     CK(cudaMalloc(&c->d_spl, sizeof(u64) * SS_MAX_LEVELS * MAX_B));
     CK(cudaMalloc(&c->d_eq, (size_t)SS_MAX_LEVELS * MAX_B));
@@ -251,6 +284,9 @@ ss_status ensure_small(ss_context* c) {
     CK(cudaHostAlloc(&c->h_res, sizeof(SelectResult), cudaHostAllocMapped));
     std::memset(c->h_res, 0, sizeof(SelectResult));
     CK(cudaHostGetDevicePointer((void**)&c->h_res_dev, c->h_res, 0));
+    CK(cudaMalloc(&c->d_seq, sizeof(u32)));
+    CK(cudaMemset(c->d_seq, 0, sizeof(u32)));
+    CK(cudaStreamCreateWithFlags(&c->cap_st, cudaStreamNonBlocking));
     return SS_OK;
 }
 
@@ -279,14 +315,18 @@ size_t res_bytes(const ss_context* c) {
 // Enqueue the result hand-off and wait for it: the publish kernel writes the
 // result block into the mapped host mirror and then the new sequence number;
 // the host spins on that word (checking the stream for errors now and then).
-ss_status publish_and_wait(ss_context* c, cudaStream_t st) {
-    const u32 seq = ++c->seq;
+ss_status enqueue_publish(ss_context* c, cudaStream_t st) {
     const u32 nwords = (u32)(res_bytes(c) / 4);
     const u32 seq_word = (u32)(offsetof(SelectResult, seq) / 4);
     CK(launch_pdl(publish_kernel, dim3(1), dim3(128), 0, st, reinterpret_cast<const u32*>(c->d_res),
-                  reinterpret_cast<u32*>(c->h_res_dev), nwords, seq_word, seq));
+                  reinterpret_cast<u32*>(c->h_res_dev), nwords, seq_word, c->d_seq));
     CKLAUNCH("publish_kernel");
     ++c->launches;
+    return SS_OK;
+}
+
+ss_status wait_publish(ss_context* c, cudaStream_t st) {
+    const u32 seq = ++c->seq;
     c->d2h += res_bytes(c);
     volatile u32* flag = &c->h_res->seq;
     for (u64 spin = 1;; ++spin) {
@@ -399,28 +439,34 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     for (int i = 0; i < 2; ++i)
         if ((rc = grow(c, &c->d_buf[i], &c->cap_buf[i], n * sizeof(T)))) return rc;
     int L = expected_levels(n, b0, bd, B);
-    // totals of every level are zeroed here; levels beyond the plan (the
-    // rare "incomplete" fallback) are zeroed before they run
     // level 0's sample is gathered by the init kernel when the wide K1 ranks it
     const bool pre0 = L > 0 && s <= WIDE_K1_MAX_S;
     K* sample0 = pre0 ? reinterpret_cast<K*>(c->d_sample0) : nullptr;
-    CK(launch_pdl(init_kernel<T>, dim3(pre0 ? (u32)s / 256u : 1u), dim3(256), 0, st, c->d_ctl,
-                  (int)(SS_MAX_LEVELS + 1), c->d_totals, (int)((L + 1) * MAX_B), c->d_res, n, k,
-                  (int)(c->cfg.profile == 3), d, s, (u64)c->cfg.seed, sample0));
-    CKLAUNCH("init_kernel");
-    ++c->launches;
-    int lev = 0;
-    const T* in = d;
-    for (;;) {
+    const int tl_on = c->cfg.profile == 3;
+    // totals of every planned level are zeroed by init; levels beyond the plan
+    // (the rare "incomplete" fallback) are zeroed before they run
+    auto enqueue_init = [&](cudaStream_t q) -> ss_status {
+        CK(launch_pdl(init_kernel<T>, dim3(pre0 ? (u32)s / 256u : 1u), dim3(256), 0, q, c->d_ctl,
+                      (int)(SS_MAX_LEVELS + 1), c->d_totals, (int)((L + 1) * MAX_B), c->d_res, n, k, tl_on, d, s,
+                      (u64)c->cfg.seed, sample0));
+        CKLAUNCH("init_kernel");
+        ++c->launches;
+        return SS_OK;
+    };
+    // levels [lev0, L) and the final K1 (base case or "incomplete" flag)
+    auto enqueue_levels = [&](int lev0, cudaStream_t q) -> ss_status {
+        ss_status rc2;
+        const T* in = lev0 ? reinterpret_cast<const T*>(c->d_buf[(lev0 - 1) & 1]) : d;
+        int lev = lev0;
         for (; lev < L; ++lev) {
             const int b = lev ? bd : b0, H = log2i(b);
             const u32 grid = grid_for<T>(c, H);
             const int sl = lev ? s_deep : s;
             const bool wide = sl <= WIDE_K1_MAX_S;
             if (wide) {
-                if ((rc = launch_k1_wide<T>(c, in, lev, sl, B, st, lev == 0 ? sample0 : nullptr))) return rc;
-            } else if ((rc = launch_k1<T>(c, in, lev, sl, b, 1, B, 0, st))) {
-                return rc;
+                if ((rc2 = launch_k1_wide<T>(c, in, lev, sl, B, q, lev == 0 ? sample0 : nullptr))) return rc2;
+            } else if ((rc2 = launch_k1<T>(c, in, lev, sl, b, 1, B, 0, q))) {
+                return rc2;
             }
             CountArgs a{};
             if (wide) {
@@ -438,12 +484,11 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             a.cta_counts = c->d_cta_counts;
             a.warp_counts = c->d_warp_counts;
             a.totals = c->d_totals + (size_t)lev * MAX_B;
-            a.offsets = c->d_offsets;
             a.level = lev;
             a.tail = TAIL_EXACT;
-            mark(c, lev, 1, 0, st);
-            if ((rc = launch_count<T>(c, H, in, a, st))) return rc;
-            mark(c, lev, 1, 1, st);
+            mark(c, lev, 1, 0, q);
+            if ((rc2 = launch_count<T>(c, H, in, a, q))) return rc2;
+            mark(c, lev, 1, 1, q);
             ++c->launches;
             if (a.grid != grid) return fail(c, SS_ERR_INTERNAL, "grid mismatch");
             T* out = reinterpret_cast<T*>(c->d_buf[lev & 1]);
@@ -451,26 +496,132 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             f.ctl = c->d_ctl + lev;
             f.res = c->d_res;
             f.oracles = c->d_oracles;
-            f.offsets = c->d_offsets;
+            f.cta_counts = c->d_cta_counts;
             f.warp_counts = c->d_warp_counts;
             f.b_count = (u32)b;
             f.grid = grid;
             f.level = lev;
-            mark(c, lev, 2, 0, st);
-            CK(launch_pdl(filter_kernel<T>, dim3(grid), dim3(K5_THREADS), FILTER_SMEM, st, in, out, f));
+            mark(c, lev, 2, 0, q);
+            CK(launch_pdl(filter_kernel<T>, dim3(grid), dim3(K5_THREADS), FILTER_SMEM, q, in, out, f));
             CKLAUNCH("filter_kernel");
-            mark(c, lev, 2, 1, st);
+            mark(c, lev, 2, 1, q);
             ++c->launches;
             in = out;
         }
-        if ((rc = launch_k1<T>(c, in, lev, lev ? s_deep : s, lev ? bd : b0, 1, B, 1, st))) return rc;
-        if ((rc = publish_and_wait(c, st))) return rc;
-        if (c->h_res->done) break;
-        if (!c->h_res->incomplete || lev >= SS_MAX_LEVELS - 2)
+        return launch_k1<T>(c, in, lev, lev ? s_deep : s, lev ? bd : b0, 1, B, 1, q);
+    };
+    // the planned part of the call: one CUDA graph launch (events of
+    // profile 1/2 cannot live in a graph: those calls launch directly)
+    const bool graph = c->use_graphs && c->cfg.profile != 1 && c->cfg.profile != 2;
+    ss_context::GraphEntry* ge = nullptr;
+    if (graph) {
+        for (auto& e : c->graphs)
+            if (e.used && e.dt == dt_code<T>() && e.ptr == d &&
+                e.n == n && e.b0 == b0 && e.bd == bd && e.s == s && e.sd == s_deep && e.L == L &&
+                e.prof == tl_on && e.B == B && e.seed == c->cfg.seed)
+                ge = &e;
+        if (!ge) {
+            ss_context::GraphEntry* slot = nullptr;           // a free entry, else the least recently used
+            for (auto& e : c->graphs)
+                if (!e.used) { slot = &e; break; }
+            if (!slot) {
+                slot = &c->graphs[0];
+                for (auto& e : c->graphs)
+                    if (e.stamp < slot->stamp) slot = &e;
+            }
+            if (slot->exec) cudaGraphExecDestroy(slot->exec);
+            if (slot->graph) cudaGraphDestroy(slot->graph);
+            *slot = ss_context::GraphEntry();
+            const int launches0 = c->launches;
+            CK(cudaStreamBeginCapture(c->cap_st, cudaStreamCaptureModeThreadLocal));
+            ss_status rc2 = enqueue_init(c->cap_st);
+            if (!rc2) rc2 = enqueue_levels(0, c->cap_st);
+            if (!rc2) rc2 = enqueue_publish(c, c->cap_st);
+            cudaGraph_t g = nullptr;
+            const cudaError_t ec = cudaStreamEndCapture(c->cap_st, &g);
+            if (rc2) {
+                if (g) cudaGraphDestroy(g);
+                return rc2;
+            }
+            CK(ec);
+            cudaGraphExec_t ex = nullptr;
+            const cudaError_t ei = cudaGraphInstantiate(&ex, g, 0);
+            // the init node: the graph's only kernel node running init_kernel<T>
+            size_t nn = 0;
+            cudaGraphGetNodes(g, nullptr, &nn);
+            std::vector<cudaGraphNode_t> nodes(nn);
+            cudaGraphGetNodes(g, nodes.data(), &nn);
+            cudaGraphNode_t init_node = nullptr;
+            cudaKernelNodeParams ip{};
+            for (auto nd : nodes) {
+                cudaGraphNodeType ty;
+                cudaGraphNodeGetType(nd, &ty);
+                if (ty != cudaGraphNodeTypeKernel) continue;
+                cudaKernelNodeParams kp{};
+                if (cudaGraphKernelNodeGetParams(nd, &kp) == cudaSuccess &&
+                    kp.func == reinterpret_cast<void*>(init_kernel<T>)) {
+                    init_node = nd;
+                    ip = kp;
+                }
+            }
+            if (ei != cudaSuccess || !init_node) {
+                cudaGraphDestroy(g);
+                if (ex) cudaGraphExecDestroy(ex);
+                (void)cudaGetLastError();
+                return fail(c, SS_ERR_CUDA, "graph capture of the level chain failed");
+            }
+            slot->used = true;
+            slot->dt = dt_code<T>();
+            slot->ptr = d;
+            slot->n = n;
+            slot->b0 = b0; slot->bd = bd; slot->s = s; slot->sd = s_deep; slot->L = L;
+            slot->prof = tl_on; slot->B = B; slot->seed = c->cfg.seed;
+            slot->exec = ex;
+            slot->init_node = init_node;
+            slot->kernels = c->launches - launches0;
+            // private copy of the init arguments; k is the 7th (index 6)
+            slot->init_params = ip;
+            size_t off = 0;
+            const size_t sizes[12] = {sizeof(LevelCtl*), sizeof(int), sizeof(u64*), sizeof(int), sizeof(SelectResult*),
+                                      sizeof(u64), sizeof(u64), sizeof(int), sizeof(const T*), sizeof(int), sizeof(u64),
+                                      sizeof(K*)};
+            for (int i = 0; i < 12; ++i) {
+                off = (off + 7) & ~(size_t)7;
+                std::memcpy(slot->init_store + off, ip.kernelParams[i], sizes[i]);
+                slot->init_args[i] = slot->init_store + off;
+                if (i == 6) slot->k_offset = off;
+                off += sizes[i];
+            }
+            slot->init_params.kernelParams = slot->init_args;
+            slot->init_params.extra = nullptr;
+            slot->graph = g;
+            ge = slot;
+            c->launches = launches0;
+        } else {
+            u64 kk = k;
+            std::memcpy(ge->init_store + ge->k_offset, &kk, sizeof(u64));
+            CK(cudaGraphExecKernelNodeSetParams(ge->exec, ge->init_node, &ge->init_params));
+        }
+        ge->stamp = ++c->graph_clock;
+        CK(cudaGraphLaunch(ge->exec, st));
+        c->launches += ge->kernels;
+    } else {
+        if ((rc = enqueue_init(st))) return rc;
+        if ((rc = enqueue_levels(0, st))) return rc;
+        if ((rc = enqueue_publish(c, st))) return rc;
+    }
+    if ((rc = wait_publish(c, st))) return rc;
+    // rare: an unlucky sample left more than B elements after the planned levels
+    while (!c->h_res->done) {
+        if (!c->h_res->incomplete || L >= SS_MAX_LEVELS - 2)
             return fail(c, SS_ERR_INTERNAL, "recursion did not terminate");
         CK(cudaMemsetAsync(&c->d_res->incomplete, 0, sizeof(int), st));
-        L = lev + 1;
-        CK(cudaMemsetAsync(c->d_totals + (size_t)lev * MAX_B, 0, sizeof(u64) * MAX_B, st));
+        CK(cudaMemsetAsync(c->d_totals + (size_t)L * MAX_B, 0, sizeof(u64) * MAX_B, st));
+        const int lev0 = L;
+        L = L + 1;
+        if ((rc = enqueue_levels(lev0, st))) return rc;
+        if ((rc = enqueue_publish(c, st))) return rc;
+        if ((rc = wait_publish(c, st))) return rc;
     }
     const SelectResult& r = *c->h_res;
     std::memcpy(h_result, &r.bits, sizeof(T));
@@ -539,14 +690,14 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     a.oracles = nullptr;
     a.cta_counts = nullptr;
     a.totals = c->d_totals;
-    a.offsets = nullptr;
     a.level = 0;
     a.tail = TAIL_APPROX;
     mark(c, 0, 1, 0, st);
     if ((rc = launch_count<T>(c, H, d, a, st))) return rc;
     mark(c, 0, 1, 1, st);
     ++c->launches;
-    if ((rc = publish_and_wait(c, st))) return rc;
+    if ((rc = enqueue_publish(c, st))) return rc;
+    if ((rc = wait_publish(c, st))) return rc;
     const SelectResult& r = *c->h_res;
     if (!r.done) return fail(c, SS_ERR_INTERNAL, "approximate select produced no result");
     std::memcpy(h_result, &r.bits, sizeof(T));
@@ -662,12 +813,17 @@ void ss_destroy(ss_context* c) {
     cudaFree(c->d_totals);
     cudaFree(c->d_cta_counts);
     cudaFree(c->d_warp_counts);
-    cudaFree(c->d_offsets);
     cudaFree(c->d_tree);
     cudaFree(c->d_spl);
     cudaFree(c->d_eq);
     cudaFree(c->d_sorted);
     cudaFree(c->d_sample0);
+    cudaFree(c->d_seq);
+    for (auto& e : c->graphs) {
+        if (e.exec) cudaGraphExecDestroy(e.exec);
+        if (e.graph) cudaGraphDestroy(e.graph);
+    }
+    if (c->cap_st) cudaStreamDestroy(c->cap_st);
     if (c->h_res) cudaFreeHost(c->h_res);
     if (c->ev_ready)
         for (int l = 0; l < SS_MAX_LEVELS; ++l)
@@ -698,7 +854,14 @@ ss_status ss_set_config(ss_context* c, const ss_config* cfg) {
         return fail(c, SS_ERR_INVALID_ARGUMENT, "profile must be 0, 1, 2 or 3");
     if (cfg->ctas_per_sm < 1 || cfg->ctas_per_sm > 16)
         return fail(c, SS_ERR_INVALID_ARGUMENT, "ctas_per_sm must be in [1, 16]");
+    const bool regrid = cfg->ctas_per_sm != c->cfg.ctas_per_sm;
     c->cfg = *cfg;
+    if (regrid)                   // captured grid sizes are stale (the other knobs are part of the graph key)
+        for (auto& e : c->graphs) {
+            if (e.exec) cudaGraphExecDestroy(e.exec);
+            if (e.graph) cudaGraphDestroy(e.graph);
+            e = ss_context::GraphEntry();
+        }
     return SS_OK;
 }
 
@@ -876,13 +1039,10 @@ ss_status ss_step_filter(ss_context* c, ss_dtype dt, const void* d_data, int64_t
     const u32 grid = c->step_grid;
     return dispatch(dt, [&](auto* tag) -> ss_status {
         typedef std::remove_pointer_t<decltype(tag)> T;
-        Chunking ch = make_chunking((const T*)d_data, (u64)n, grid);
-        offsets_kernel<<<1, 1024, 0, st>>>(c->d_cta_counts, (u32)c->step_b, (u32)bucket, ch.ncta, c->d_offsets);
-        CKLAUNCH("offsets_kernel");
         CK(cudaMemsetAsync(d_count, 0, sizeof(u64), st));
         FilterArgs f{};
         f.oracles = d_oracles;
-        f.offsets = c->d_offsets;
+        f.cta_counts = c->d_cta_counts;
         f.warp_counts = c->d_warp_counts;
         f.b_count = (u32)c->step_b;
         f.count_out = (u64*)d_count;

@@ -25,10 +25,14 @@ acc = None
 for _ in range(R):
     run()
     st = ctx.stats()
-    tl = np.array(st["tl_us"], dtype=np.float64)
+    tl = np.array(ctx.raw_tl() if os.environ.get("TL_DEBUG") else st["tl_us"], dtype=np.float64)
     acc = tl if acc is None else acc + tl
 tl = acc / R
 names = ["K1", "K2", "K5"]
+if os.environ.get("TL_DEBUG"):
+    for sl, nm in ((93, "L1K2 cta start"), (90, "L1K2 prologue end"), (91, "L1K2 main end"), (92, "L1K2 ticket")):
+        l, q = divmod(sl, 3)
+        print(f"  {nm}: first {tl[l][q][0]:8.1f}  last {tl[l][q][1]:8.1f}")
 print(f"n=2^{log2n} b={b} b_deep={bd} {mode}: n_level={st['n_level']}  (mean of {R} calls, us after init)")
 for l in range(tl.shape[0]):
     for q in range(3):
