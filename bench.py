@@ -48,6 +48,7 @@ def parse():
     p.add_argument("--e2e-steps", type=int, default=0, help="host-buffer steps (default: min(steps, 10))")
     p.add_argument("--cpu-seconds", type=float, default=10.0, help="CPU-oracle baseline budget")
     p.add_argument("--no-cpu", action="store_true")
+    p.add_argument("--classify", type=int, default=0, help="0 auto (cell LUT where it applies), 1 tree walk")
     p.add_argument("--events", default="separate", choices=["timed", "separate"],
                    help="CUDA events around K2 inside the timed loop (timed: they break the PDL overlap "
                         "of the kernel chain) or in a second timed pass of the same length (separate)")
@@ -219,6 +220,8 @@ def run_ours(args, rank, world, local_rank):
     xd = xh.to(f"cuda:{dev}", non_blocking=False)
     torch.cuda.synchronize()
     ctx = ss.Context(dev)
+    if args.classify:
+        ctx.configure(classify=args.classify)
     exact = args.mode == "exact"
     b = args.b or (256 if exact else 1024)
     if exact:

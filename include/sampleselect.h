@@ -37,7 +37,7 @@
 extern "C" {
 #endif
 
-#define SS_ABI_VERSION 1
+#define SS_ABI_VERSION 2
 #define SS_MAX_LEVELS 32
 
 typedef enum { SS_FLOAT32 = 0, SS_FLOAT64 = 1, SS_INT32 = 2, SS_INT64 = 3 } ss_dtype;
@@ -68,6 +68,10 @@ typedef struct {
     int32_t b_deep;       /* buckets of the levels after the first: 0 = b_exact, else a
                              power of two in [4, 256] (each level is a full SampleSelect
                              level of Fig. 1; only its bucket count differs) */
+    int32_t classify;     /* bucket classification in the count kernel: 0 = auto (cell
+                             lookup table for 4-byte keys and b <= 256 where its
+                             marker cells are light, else the Fig. 4 tree walk);
+                             1 = always the tree walk.  Same buckets either way. default 0 */
     uint64_t seed;        /* sampling seed (reading R7). default 0x5A17 */
 } ss_config;
 
@@ -88,6 +92,10 @@ typedef struct {
                                           us after the call's init kernel, from %globaltimer
                                           stamps taken inside the kernels (no events, so the
                                           PDL overlap of the chain is kept); -1 = not run */
+    int32_t lut_ctas;                  /* level-0 count CTAs that classified with the cell
+                                          lookup table (0 = all walked the tree) */
+    int32_t lut_marker;                /* level 0: whole buckets inside the table's marker
+                                          cells (the auto rule walks the tree when >= 2) */
 } ss_stats;
 
 /* ---- context --------------------------------------------------------- */

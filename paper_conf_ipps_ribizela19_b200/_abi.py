@@ -31,7 +31,7 @@ class SSConfig(ctypes.Structure):
     _fields_ = [("b_exact", ctypes.c_int32), ("sample_size", ctypes.c_int32),
                 ("base_case", ctypes.c_int32), ("ctas_per_sm", ctypes.c_int32),
                 ("profile", ctypes.c_int32), ("b_deep", ctypes.c_int32),
-                ("seed", ctypes.c_uint64)]
+                ("classify", ctypes.c_int32), ("seed", ctypes.c_uint64)]
 
 
 class SSStats(ctypes.Structure):
@@ -42,7 +42,8 @@ class SSStats(ctypes.Structure):
                 ("launches", ctypes.c_int32),
                 ("h2d_bytes", ctypes.c_int64), ("d2h_bytes", ctypes.c_int64),
                 ("ms_kernel", (ctypes.c_float * 3) * SS_MAX_LEVELS),
-                ("tl_us", ((ctypes.c_float * 2) * 3) * SS_MAX_LEVELS)]
+                ("tl_us", ((ctypes.c_float * 2) * 3) * SS_MAX_LEVELS),
+                ("lut_ctas", ctypes.c_int32), ("lut_marker", ctypes.c_int32)]
 
 
 class SSError(RuntimeError):

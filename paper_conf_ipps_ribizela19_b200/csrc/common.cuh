@@ -66,7 +66,7 @@ struct LevelCtl {
     u32 ticket;     // count-kernel CTA completion ticket (last CTA runs the tail)
     u32 bucket;     // bucket j chosen at level l
     u32 ncta;       // active CTAs of the count/filter grid
-    u32 pad;
+    u32 marker;     // whole buckets inside the cell LUT's marker cells (tree_image_kernel)
 };
 
 struct SelectResult {
@@ -79,6 +79,7 @@ struct SelectResult {
     long long n_level[32];
     int bucket[32];
     long long split_index;    // approximate: 1-based splitter index returned
+    unsigned int lut_stats[2];// level 0: CTAs that used the cell LUT, marker-cell buckets
     unsigned int seq;         // host mirror only: publish sequence number, written last
     int pad_seq;
     int tl_on;                // timeline mode (profile = 3): kernels stamp tl[]
@@ -111,20 +112,19 @@ struct TimelineScope {
 };
 
 // ------------------------------------------------------------ chunking ----
-// Element -> unit mapping shared by the count (K2) and filter (K5) kernels;
+// Element -> CTA mapping shared by the count (K2) and filter (K5) kernels;
 // the filter must see exactly the count's partition so that the K3 offsets
 // apply (§IV.G).  The body is cut into 16-element groups (16 oracle
-// bytes = one 128-bit load); a "unit" is the contiguous run of groups owned
-// by one warp: unit u = g * UNIT_WARPS + w owns groups [u*gpw, (u+1)*gpw).
-// Elements [0, head) are peeled so the body starts 16-byte aligned (unit 0
-// owns them); [tail_begin, n) (< 16 elements) belongs to the last unit of the
-// last active CTA.  K2 counts per unit; K5 compacts per unit with no
-// cross-warp synchronisation.
-constexpr u32 UNIT_WARPS = 16;          // warps per CTA in K2 and K5 (512 threads)
-constexpr u64 MIN_GROUPS_PER_UNIT = 4;  // 64 elements: small levels still spread over many warps
+// bytes = one 128-bit load); CTA g owns the contiguous groups
+// [g*gpc, (g+1)*gpc).  Elements [0, head) are peeled so the body starts
+// 16-byte aligned (CTA 0 owns them); [tail_begin, n) (< 16 elements) belongs
+// to the last active CTA.  Inside its chunk K2 gives each warp a contiguous
+// run of groups (any order counts the same); K5 walks the chunk in slices so
+// that its output is in input order (reading R15).
+constexpr u64 MIN_GROUPS_PER_CTA = 32;  // 512 elements: small levels still spread over many CTAs
 
 struct Chunking {
-    u64 head, ngroups, tail_begin, gpw;
+    u64 head, ngroups, tail_begin, gpc;
     u32 ncta;
 };
 
@@ -137,12 +137,10 @@ __host__ __device__ __forceinline__ Chunking make_chunking(const T* p, u64 n, u3
     c.head = head;
     c.ngroups = (n - head) / 16;
     c.tail_begin = head + c.ngroups * 16;
-    const u64 units_max = (u64)grid * UNIT_WARPS;
-    u64 gpw = (c.ngroups + units_max - 1) / units_max;
-    if (gpw < MIN_GROUPS_PER_UNIT) gpw = MIN_GROUPS_PER_UNIT;
-    c.gpw = gpw;
-    const u64 units = (c.ngroups + gpw - 1) / gpw;
-    u64 nc = (units + UNIT_WARPS - 1) / UNIT_WARPS;
+    u64 gpc = (c.ngroups + grid - 1) / grid;
+    if (gpc < MIN_GROUPS_PER_CTA) gpc = MIN_GROUPS_PER_CTA;
+    c.gpc = gpc;
+    u64 nc = (c.ngroups + gpc - 1) / gpc;
     if (nc == 0) nc = 1;
     if (nc > grid) nc = grid;
     c.ncta = (u32)nc;

@@ -41,12 +41,12 @@ struct ss_context {
     SelectResult* d_res = nullptr;
     u64* d_totals = nullptr;     // [SS_MAX_LEVELS][MAX_B]
     u32* d_cta_counts = nullptr; // [MAX_GRID][MAX_B]
-    u32* d_warp_counts = nullptr; // [MAX_GRID][UNIT_WARPS][256]
     u64* d_tree = nullptr;       // [SS_MAX_LEVELS][MAX_B] keys (u32 keys use the same bytes)
     u64* d_spl = nullptr;
     uint8_t* d_eq = nullptr;     // [SS_MAX_LEVELS][MAX_B]
     u64* d_sorted = nullptr;     // [SS_MAX_LEVELS][MAX_S] sorted sample keys (wide K1)
     u64* d_sample0 = nullptr;    // [MAX_S] level-0 sample keys (gathered by the init kernel)
+    uint8_t* d_image = nullptr;  // [SS_MAX_LEVELS][K2_IMAGE_SLOT] count-kernel images (tree_image_kernel)
     SelectResult* h_res = nullptr;   // mapped pinned mirror of d_res (written by publish_kernel)
     SelectResult* h_res_dev = nullptr;
     u32 seq = 0;                     // publishes issued (host count, lockstep with *d_seq)
@@ -93,6 +93,9 @@ struct ss_context {
 };
 
 static constexpr u32 MAX_GRID = 2048;
+// SS_CARVEOUT (build flag): force one shared-memory carveout on every kernel
+// of the chain.  Off by default: measured slower -- an all-shared carveout
+// leaves L1 too small for the count kernel's in-flight 128-bit loads.
 static constexpr int MAX_S = 16384;
 // sample sizes up to this are ranked by the wide K1 (s/32 CTAs, s^2 pairs);
 // larger samples (approximate b = 1024) use the one-CTA bitonic K1
@@ -265,6 +268,8 @@ ss_status set_k1_attrs(ss_context* c) {
 #ifdef SS_CARVEOUT
     CK(cudaFuncSetAttribute(sample_tree_kernel<T>, cudaFuncAttributePreferredSharedMemoryCarveout, SS_CARVEOUT));
     CK(cudaFuncSetAttribute(filter_kernel<T>, cudaFuncAttributePreferredSharedMemoryCarveout, SS_CARVEOUT));
+    CK(cudaFuncSetAttribute(sample_rank_kernel<T>, cudaFuncAttributePreferredSharedMemoryCarveout, SS_CARVEOUT));
+    CK(cudaFuncSetAttribute(init_kernel<T>, cudaFuncAttributePreferredSharedMemoryCarveout, SS_CARVEOUT));
 #endif
     return SS_OK;
 }
@@ -275,12 +280,12 @@ ss_status ensure_small(ss_context* c) {
     CK(cudaMalloc(&c->d_res, sizeof(SelectResult)));
     CK(cudaMalloc(&c->d_totals, sizeof(u64) * SS_MAX_LEVELS * MAX_B));
     CK(cudaMalloc(&c->d_cta_counts, sizeof(u32) * (size_t)MAX_GRID * MAX_B));
-    CK(cudaMalloc(&c->d_warp_counts, sizeof(u32) * (size_t)MAX_GRID * UNIT_WARPS * 256));
     CK(cudaMalloc(&c->d_tree, sizeof(u64) * SS_MAX_LEVELS * MAX_B));
     CK(cudaMalloc(&c->d_spl, sizeof(u64) * SS_MAX_LEVELS * MAX_B));
     CK(cudaMalloc(&c->d_eq, (size_t)SS_MAX_LEVELS * MAX_B));
     CK(cudaMalloc(&c->d_sorted, sizeof(u64) * SS_MAX_LEVELS * MAX_S));
     CK(cudaMalloc(&c->d_sample0, sizeof(u64) * MAX_S));
+    CK(cudaMalloc(&c->d_image, K2_IMAGE_SLOT * SS_MAX_LEVELS));
     CK(cudaHostAlloc(&c->h_res, sizeof(SelectResult), cudaHostAllocMapped));
     std::memset(c->h_res, 0, sizeof(SelectResult));
     CK(cudaHostGetDevicePointer((void**)&c->h_res_dev, c->h_res, 0));
@@ -418,6 +423,32 @@ ss_status launch_k1_wide(ss_context* c, const T* in, int lev, int s, u32 B, cuda
     return SS_OK;
 }
 
+// K1b: the level's tree + count-kernel image from the wide K1's sorted sample.
+template <typename T>
+ss_status launch_image(ss_context* c, int H, int lev, int s, int fixup, cudaStream_t st) {
+    typedef typename Traits<T>::Key K;
+    const K* sorted = reinterpret_cast<const K*>(c->d_sorted) + (size_t)lev * MAX_S;
+    uint8_t* image = c->d_image + (size_t)lev * K2_IMAGE_SLOT;
+    K* tree = reinterpret_cast<K*>(c->d_tree) + (size_t)lev * MAX_B;
+    K* spl = reinterpret_cast<K*>(c->d_spl) + (size_t)lev * MAX_B;
+    uint8_t* eq = c->d_eq + (size_t)lev * MAX_B;
+    const int lut_on = c->cfg.classify == 0;
+#define SS_IMG_CASE(h)                                                                                     \
+    case h:                                                                                                \
+        CK(launch_pdl(tree_image_kernel<T, h>, dim3(IMG_CTAS), dim3(1024), 0, st, sorted, s, fixup, lut_on, \
+                      c->d_ctl + lev, c->d_res, image, tree, spl, eq));                                    \
+        break;
+    switch (H) {
+        SS_IMG_CASE(2) SS_IMG_CASE(3) SS_IMG_CASE(4) SS_IMG_CASE(5) SS_IMG_CASE(6)
+        SS_IMG_CASE(7) SS_IMG_CASE(8) SS_IMG_CASE(9) SS_IMG_CASE(10)
+    default: return fail(c, SS_ERR_INVALID_ARGUMENT, "b must be a power of two in [4, 1024]");
+    }
+#undef SS_IMG_CASE
+    CKLAUNCH("tree_image_kernel");
+    ++c->launches;
+    return SS_OK;
+}
+
 template <typename T>
 ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cudaStream_t st) {
     typedef typename Traits<T>::Key K;
@@ -465,15 +496,12 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             const bool wide = sl <= WIDE_K1_MAX_S;
             if (wide) {
                 if ((rc2 = launch_k1_wide<T>(c, in, lev, sl, B, q, lev == 0 ? sample0 : nullptr))) return rc2;
+                if ((rc2 = launch_image<T>(c, H, lev, sl, 1, q))) return rc2;
             } else if ((rc2 = launch_k1<T>(c, in, lev, sl, b, 1, B, 0, q))) {
                 return rc2;
             }
             CountArgs a{};
-            if (wide) {
-                a.sorted = reinterpret_cast<K*>(c->d_sorted) + (size_t)lev * MAX_S;
-                a.s = sl;
-                a.fixup = 1;
-            }
+            if (wide) a.image = c->d_image + (size_t)lev * K2_IMAGE_SLOT;
             a.ctl = c->d_ctl + lev;
             a.ctl_next = c->d_ctl + lev + 1;
             a.res = c->d_res;
@@ -482,8 +510,9 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             a.eq = c->d_eq + (size_t)lev * MAX_B;
             a.oracles = c->d_oracles;
             a.cta_counts = c->d_cta_counts;
-            a.warp_counts = c->d_warp_counts;
             a.totals = c->d_totals + (size_t)lev * MAX_B;
+            a.lut = c->cfg.classify == 0;
+            a.lut_stats = lev == 0 ? c->d_res->lut_stats : nullptr;
             a.level = lev;
             a.tail = TAIL_EXACT;
             mark(c, lev, 1, 0, q);
@@ -497,7 +526,6 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             f.res = c->d_res;
             f.oracles = c->d_oracles;
             f.cta_counts = c->d_cta_counts;
-            f.warp_counts = c->d_warp_counts;
             f.b_count = (u32)b;
             f.grid = grid;
             f.level = lev;
@@ -629,6 +657,8 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     std::memset(&S, 0, sizeof(S));
     S.levels = r.levels;
     S.equality_exit = r.eq_exit;
+    S.lut_ctas = (int32_t)r.lut_stats[0];
+    S.lut_marker = (int32_t)r.lut_stats[1];
     double bytes = 0;
     const double Sz = (double)sizeof(T);
     for (int l = 0; l <= r.levels && l < SS_MAX_LEVELS; ++l) {
@@ -672,15 +702,12 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     ++c->launches;
     if (wide) {
         if ((rc = launch_k1_wide<T>(c, d, 0, s, 0, st, sample0))) return rc;
+        if ((rc = launch_image<T>(c, H, 0, s, 0, st))) return rc;
     } else if ((rc = launch_k1<T>(c, d, 0, s, b, 0, 0, 0, st))) {
         return rc;
     }
     CountArgs a{};
-    if (wide) {
-        a.sorted = reinterpret_cast<K*>(c->d_sorted);
-        a.s = s;
-        a.fixup = 0;
-    }
+    if (wide) a.image = c->d_image;
     a.ctl = c->d_ctl;
     a.ctl_next = c->d_ctl + 1;
     a.res = c->d_res;
@@ -690,6 +717,8 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     a.oracles = nullptr;
     a.cta_counts = nullptr;
     a.totals = c->d_totals;
+    a.lut = c->cfg.classify == 0;
+    a.lut_stats = c->d_res->lut_stats;
     a.level = 0;
     a.tail = TAIL_APPROX;
     mark(c, 0, 1, 0, st);
@@ -705,6 +734,8 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     ss_stats& S = c->stats;
     std::memset(&S, 0, sizeof(S));
     S.levels = 1;
+    S.lut_ctas = (int32_t)r.lut_stats[0];
+    S.lut_marker = (int32_t)r.lut_stats[1];
     S.n_level[0] = (int64_t)n;
     S.bucket[0] = (int32_t)r.split_index;
     S.bytes_algorithmic = (double)sizeof(T) * (double)n;
@@ -782,6 +813,7 @@ ss_status ss_create(int device, ss_context** out) {
     c->cfg.ctas_per_sm = 4;
     c->cfg.profile = 0;
     c->cfg.seed = 0x5A17;
+    c->cfg.classify = 0;
     DevGuard g(device);
     if (cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess) {
         (void)cudaGetLastError();
@@ -812,12 +844,12 @@ void ss_destroy(ss_context* c) {
     cudaFree(c->d_res);
     cudaFree(c->d_totals);
     cudaFree(c->d_cta_counts);
-    cudaFree(c->d_warp_counts);
     cudaFree(c->d_tree);
     cudaFree(c->d_spl);
     cudaFree(c->d_eq);
     cudaFree(c->d_sorted);
     cudaFree(c->d_sample0);
+    cudaFree(c->d_image);
     cudaFree(c->d_seq);
     for (auto& e : c->graphs) {
         if (e.exec) cudaGraphExecDestroy(e.exec);
@@ -852,9 +884,11 @@ ss_status ss_set_config(ss_context* c, const ss_config* cfg) {
         return fail(c, SS_ERR_INVALID_ARGUMENT, "base_case must be a power of two in [256, 16384]");
     if (cfg->profile < 0 || cfg->profile > 3)
         return fail(c, SS_ERR_INVALID_ARGUMENT, "profile must be 0, 1, 2 or 3");
+    if (cfg->classify < 0 || cfg->classify > 1)
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "classify must be 0 (auto) or 1 (tree walk)");
     if (cfg->ctas_per_sm < 1 || cfg->ctas_per_sm > 16)
         return fail(c, SS_ERR_INVALID_ARGUMENT, "ctas_per_sm must be in [1, 16]");
-    const bool regrid = cfg->ctas_per_sm != c->cfg.ctas_per_sm;
+    const bool regrid = cfg->ctas_per_sm != c->cfg.ctas_per_sm || cfg->classify != c->cfg.classify;
     c->cfg = *cfg;
     if (regrid)                   // captured grid sizes are stale (the other knobs are part of the graph key)
         for (auto& e : c->graphs) {
@@ -1012,8 +1046,8 @@ ss_status ss_step_count(ss_context* c, ss_dtype dt, const void* d_data, int64_t 
         a.tree = d_tree;
         a.oracles = d_oracles;
         a.cta_counts = c->d_cta_counts;
-        a.warp_counts = b <= 256 ? c->d_warp_counts : nullptr;
         a.totals = (u64*)d_totals;
+        a.lut = c->cfg.classify == 0;
         a.n = (u64)n;
         a.tail = TAIL_NONE;
         ss_status r2 = launch_count<T>(c, log2i(b), (const T*)d_data, a, st);
@@ -1043,7 +1077,6 @@ ss_status ss_step_filter(ss_context* c, ss_dtype dt, const void* d_data, int64_t
         FilterArgs f{};
         f.oracles = d_oracles;
         f.cta_counts = c->d_cta_counts;
-        f.warp_counts = c->d_warp_counts;
         f.b_count = (u32)c->step_b;
         f.count_out = (u64*)d_count;
         f.n = (u64)n;
