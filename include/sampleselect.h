@@ -37,7 +37,7 @@
 extern "C" {
 #endif
 
-#define SS_ABI_VERSION 2
+#define SS_ABI_VERSION 3
 #define SS_MAX_LEVELS 32
 
 typedef enum { SS_FLOAT32 = 0, SS_FLOAT64 = 1, SS_INT32 = 2, SS_INT64 = 3 } ss_dtype;
@@ -73,6 +73,18 @@ typedef struct {
                              marker cells are light, else the Fig. 4 tree walk);
                              1 = always the tree walk.  Same buckets either way. default 0 */
     uint64_t seed;        /* sampling seed (reading R7). default 0x5A17 */
+    int32_t fused_filter; /* exact levels: 1 = (default) fused speculative filter on levels with
+                             n_l >= spec_min_n: the sample predicts a window of buckets around
+                             rank k and the count kernel copies the window's elements to the
+                             next level while it counts (no oracle bytes, no filter pass; a
+                             miss falls back to a re-classifying filter); 0 = always the
+                             paper's oracle bytes + filter kernel (§IV.B-c).  Same answer. */
+    float spec_z;         /* window half-width in standard deviations of the sample rank of k
+                             (Binomial(s, k/n)); default 4 (miss probability ~6e-5) */
+    int64_t spec_min_n;   /* levels with at least this many elements speculate. default 2^25 */
+    float spec_max_frac;  /* speculate only if the window holds at most this fraction of the
+                             sample. default 0.25 */
+    int32_t reserved_;
 } ss_config;
 
 /* Per-call statistics of the last ss_select / ss_approx_select. */
@@ -96,6 +108,10 @@ typedef struct {
                                           lookup table (0 = all walked the tree) */
     int32_t lut_marker;                /* level 0: whole buckets inside the table's marker
                                           cells (the auto rule walks the tree when >= 2) */
+    int32_t spec_levels;               /* bit l: level l ran the fused speculative filter */
+    int32_t fused_levels;              /* bit l: ... and its window held bucket j (hit: the
+                                          captured window is level l+1; else the fallback
+                                          filter re-read level l) */
 } ss_stats;
 
 /* ---- context --------------------------------------------------------- */

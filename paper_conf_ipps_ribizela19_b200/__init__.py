@@ -102,7 +102,9 @@ class Context:
                 "bytes_algorithmic": s.bytes_algorithmic, "launches": s.launches,
                 "h2d_bytes": s.h2d_bytes, "d2h_bytes": s.d2h_bytes,
                 "ms_kernel": [list(s.ms_kernel[l]) for l in range(L + 1)],
-                "tl_us": [[list(s.tl_us[l][q]) for q in range(3)] for l in range(L + 1)]}
+                "tl_us": [[list(s.tl_us[l][q]) for q in range(3)] for l in range(L + 1)],
+                "spec_levels": s.spec_levels, "fused_levels": s.fused_levels,
+                "lut_ctas": s.lut_ctas}
 
     def raw_tl(self):
         """profile=3: the full 32x3 timeline (us after init; -1 = not stamped)."""

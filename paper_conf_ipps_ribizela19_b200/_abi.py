@@ -31,7 +31,10 @@ class SSConfig(ctypes.Structure):
     _fields_ = [("b_exact", ctypes.c_int32), ("sample_size", ctypes.c_int32),
                 ("base_case", ctypes.c_int32), ("ctas_per_sm", ctypes.c_int32),
                 ("profile", ctypes.c_int32), ("b_deep", ctypes.c_int32),
-                ("classify", ctypes.c_int32), ("seed", ctypes.c_uint64)]
+                ("classify", ctypes.c_int32), ("seed", ctypes.c_uint64),
+                ("fused_filter", ctypes.c_int32), ("spec_z", ctypes.c_float),
+                ("spec_min_n", ctypes.c_int64), ("spec_max_frac", ctypes.c_float),
+                ("reserved_", ctypes.c_int32)]
 
 
 class SSStats(ctypes.Structure):
@@ -43,7 +46,8 @@ class SSStats(ctypes.Structure):
                 ("h2d_bytes", ctypes.c_int64), ("d2h_bytes", ctypes.c_int64),
                 ("ms_kernel", (ctypes.c_float * 3) * SS_MAX_LEVELS),
                 ("tl_us", ((ctypes.c_float * 2) * 3) * SS_MAX_LEVELS),
-                ("lut_ctas", ctypes.c_int32), ("lut_marker", ctypes.c_int32)]
+                ("lut_ctas", ctypes.c_int32), ("lut_marker", ctypes.c_int32),
+                ("spec_levels", ctypes.c_int32), ("fused_levels", ctypes.c_int32)]
 
 
 class SSError(RuntimeError):

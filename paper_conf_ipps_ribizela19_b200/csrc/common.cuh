@@ -67,6 +67,19 @@ struct LevelCtl {
     u32 bucket;     // bucket j chosen at level l
     u32 ncta;       // active CTAs of the count/filter grid
     u32 marker;     // whole buckets inside the cell LUT's marker cells (tree_image_kernel)
+    // fused speculative filter: tree_image_kernel sets spec and
+    // the bucket window [wlo, whi] predicted from the sample; the count kernel
+    // then copies every element of the window to the next level's buffer
+    // (cap counts them) instead of writing oracle bytes, and its tail sets hit
+    // when the bucket holding k lies inside the window
+    u32 spec;
+    u32 wlo, whi;
+    u32 hit;
+    u64 cap;
+    u64 klo, kspan; // the window as a key range: klo <= key < klo + kspan (mod 2^bits)
+    u64 below;      // elements with key < klo (count kernel CTAs add theirs)
+    u32 nospec;     // set by a miss: this level re-runs the paper's filter on the same data
+    u32 spec_eq;    // the window is one equality bucket (§IV.C): a hit returns its value
 };
 
 struct SelectResult {
@@ -80,6 +93,10 @@ struct SelectResult {
     int bucket[32];
     long long split_index;    // approximate: 1-based splitter index returned
     unsigned int lut_stats[2];// level 0: CTAs that used the cell LUT, marker-cell buckets
+    unsigned int fused_levels;// bit l: level l's survivors came from the fused filter (window hit)
+    unsigned int spec_levels; // bit l: level l ran the fused filter (hit or miss)
+    unsigned int spec_err;    // captured count != window total (internal consistency check)
+    int pad2_;
     unsigned int seq;         // host mirror only: publish sequence number, written last
     int pad_seq;
     int tl_on;                // timeline mode (profile = 3): kernels stamp tl[]

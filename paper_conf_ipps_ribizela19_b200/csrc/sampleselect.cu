@@ -9,6 +9,7 @@
 // case (rare: an unlucky sample) more levels are enqueued.  One device->host
 // copy per call returns the answer; there is no per-level host round trip.
 #include <algorithm>
+#include <cmath>
 #include <atomic>
 #include <cstddef>
 #include <cstdlib>
@@ -231,6 +232,20 @@ ss_status launch_count(ss_context* c, int H, const T* in, CountArgs& a, cudaStre
     return SS_OK;
 }
 
+// fused-filter count kernel: one CTA per SM, KW_STASH bytes of stash
+template <typename T>
+ss_status launch_window(ss_context* c, int /*H*/, const T* in, CountArgs a, cudaStream_t st) {
+    a.grid = (u32)c->sms;
+    static bool attr_set[64] = {};
+    if (!attr_set[c->device & 63]) {
+        CK(cudaFuncSetAttribute(window_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)KW_STASH));
+        attr_set[c->device & 63] = true;
+    }
+    CK(launch_pdl(window_kernel<T>, dim3(a.grid), dim3(KW_THREADS), KW_STASH, st, in, a));
+    CKLAUNCH("window_kernel");
+    return SS_OK;
+}
+
 template <typename T>
 u32 grid_for(ss_context* c, int H) {
     switch (H) {
@@ -377,13 +392,31 @@ void prof_collect(ss_context* c) {
     (void)cudaGetLastError();
 }
 
-int expected_levels(u64 n, int b0, int bd, u32 B) {
+SpecParams spec_params(const ss_context* c) {
+    SpecParams p;
+    p.min_n = c->cfg.fused_filter ? (u64)c->cfg.spec_min_n : ~0ull;
+    p.z = c->cfg.spec_z;
+    p.max_frac = c->cfg.spec_max_frac;
+    return p;
+}
+
+int expected_levels(const ss_context* c, u64 n, int b0, int bd, int s0, int sd, u32 B, bool* spec_plan) {
     // n_{l+1} ~ n_l / b_l times the size bias of the bucket holding k (~1.1
     // for s/b = 16); plan with 1.5x slack, fall back to more levels if needed.
+    // A fused-filter level keeps its window: at most (2 (z sigma + 2) + 1) / s
+    // of the level with sigma <= sqrt(s) / 2, plus one bucket at each end.
+    const SpecParams sp = spec_params(c);
     int L = 0;
     double m = (double)n;
     while (m > (double)B && L < SS_MAX_LEVELS - 2) {
-        m = m * 1.5 / (L ? bd : b0);
+        const int b = L ? bd : b0, s = L ? sd : s0;
+        const double f = (2.0 * (sp.z * 0.5 * std::sqrt((double)s) + 2.0) + 1.0) / s;
+        const bool spec = s <= WIDE_K1_MAX_S && m >= (double)sp.min_n && f <= sp.max_frac;
+        // levels whose size may reach min_n get the fused-filter kernel
+        // enqueued (it exits unless the device-side window decision is "spec")
+        if (spec_plan) spec_plan[L] = s <= WIDE_K1_MAX_S && f <= sp.max_frac && 2.0 * m >= (double)sp.min_n &&
+                                      sp.min_n != ~0ull;
+        m = spec ? m * 1.2 * (f + 2.0 / b) : m * 1.5 / b;
         ++L;
     }
     return L;
@@ -425,7 +458,7 @@ ss_status launch_k1_wide(ss_context* c, const T* in, int lev, int s, u32 B, cuda
 
 // K1b: the level's tree + count-kernel image from the wide K1's sorted sample.
 template <typename T>
-ss_status launch_image(ss_context* c, int H, int lev, int s, int fixup, cudaStream_t st) {
+ss_status launch_image(ss_context* c, int H, int lev, int s, int fixup, cudaStream_t st, SpecParams sp) {
     typedef typename Traits<T>::Key K;
     const K* sorted = reinterpret_cast<const K*>(c->d_sorted) + (size_t)lev * MAX_S;
     uint8_t* image = c->d_image + (size_t)lev * K2_IMAGE_SLOT;
@@ -436,7 +469,7 @@ ss_status launch_image(ss_context* c, int H, int lev, int s, int fixup, cudaStre
 #define SS_IMG_CASE(h)                                                                                     \
     case h:                                                                                                \
         CK(launch_pdl(tree_image_kernel<T, h>, dim3(IMG_CTAS), dim3(1024), 0, st, sorted, s, fixup, lut_on, \
-                      c->d_ctl + lev, c->d_res, image, tree, spl, eq));                                    \
+                      c->d_ctl + lev, c->d_res, image, tree, spl, eq, sp));                                \
         break;
     switch (H) {
         SS_IMG_CASE(2) SS_IMG_CASE(3) SS_IMG_CASE(4) SS_IMG_CASE(5) SS_IMG_CASE(6)
@@ -469,7 +502,8 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     // survivor ping-pong buffers: a level's survivors never exceed its input
     for (int i = 0; i < 2; ++i)
         if ((rc = grow(c, &c->d_buf[i], &c->cap_buf[i], n * sizeof(T)))) return rc;
-    int L = expected_levels(n, b0, bd, B);
+    bool spec_plan[SS_MAX_LEVELS] = {};
+    int L = expected_levels(c, n, b0, bd, s, s_deep, B, spec_plan);
     // level 0's sample is gathered by the init kernel when the wide K1 ranks it
     const bool pre0 = L > 0 && s <= WIDE_K1_MAX_S;
     K* sample0 = pre0 ? reinterpret_cast<K*>(c->d_sample0) : nullptr;
@@ -496,7 +530,9 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             const bool wide = sl <= WIDE_K1_MAX_S;
             if (wide) {
                 if ((rc2 = launch_k1_wide<T>(c, in, lev, sl, B, q, lev == 0 ? sample0 : nullptr))) return rc2;
-                if ((rc2 = launch_image<T>(c, H, lev, sl, 1, q))) return rc2;
+                if ((rc2 = launch_image<T>(c, H, lev, sl, 1, q,
+                                           spec_plan[lev] ? spec_params(c) : SpecParams{~0ull, 0.0f, 0.0f})))
+                    return rc2;
             } else if ((rc2 = launch_k1<T>(c, in, lev, sl, b, 1, B, 0, q))) {
                 return rc2;
             }
@@ -515,7 +551,12 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             a.lut_stats = lev == 0 ? c->d_res->lut_stats : nullptr;
             a.level = lev;
             a.tail = TAIL_EXACT;
+            a.cap_out = c->d_buf[lev & 1];   // the fused filter's window copy = next level's input
             mark(c, lev, 1, 0, q);
+            if (wide && spec_plan[lev]) {             // fused filter (runs iff the window speculates)
+                if ((rc2 = launch_window<T>(c, H, in, a, q))) return rc2;
+                ++c->launches;
+            }
             if ((rc2 = launch_count<T>(c, H, in, a, q))) return rc2;
             mark(c, lev, 1, 1, q);
             ++c->launches;
@@ -659,6 +700,9 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     S.equality_exit = r.eq_exit;
     S.lut_ctas = (int32_t)r.lut_stats[0];
     S.lut_marker = (int32_t)r.lut_stats[1];
+    S.spec_levels = (int32_t)r.spec_levels;
+    S.fused_levels = (int32_t)r.fused_levels;
+    if (r.spec_err) return fail(c, SS_ERR_INTERNAL, "fused filter: captured count != window total");
     double bytes = 0;
     const double Sz = (double)sizeof(T);
     for (int l = 0; l <= r.levels && l < SS_MAX_LEVELS; ++l) {
@@ -666,10 +710,18 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
         S.bucket[l] = r.bucket[l];
     }
     for (int l = 0; l < r.levels; ++l) {
-        double nl = (double)r.n_level[l];
+        const double nl = (double)r.n_level[l], nn = (double)r.n_level[l + 1];
+        const bool last_eq = r.eq_exit && l == r.levels - 1;
+        if (r.spec_levels >> l & 1) {
+            bytes += Sz * nl;                           // count reads the level once
+            if (!last_eq) {
+                if (r.fused_levels >> l & 1) bytes += Sz * nn;           // window copy written by the count
+                else bytes += 2.0 * Sz * nl;            // miss: the level is copied and re-run
+            }
+            continue;
+        }
         bytes += Sz * nl + nl;                          // count: read + oracle write
-        bool filtered = !(r.eq_exit && l == r.levels - 1);
-        if (filtered) bytes += nl + 2.0 * Sz * (double)r.n_level[l + 1];  // oracle read + gather + write
+        if (!last_eq) bytes += nl + 2.0 * Sz * nn;      // oracle read + gather + write
     }
     if (!r.eq_exit) bytes += Sz * (double)r.n_level[r.levels];  // base case reads its input
     S.bytes_algorithmic = bytes;
@@ -702,7 +754,7 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     ++c->launches;
     if (wide) {
         if ((rc = launch_k1_wide<T>(c, d, 0, s, 0, st, sample0))) return rc;
-        if ((rc = launch_image<T>(c, H, 0, s, 0, st))) return rc;
+        if ((rc = launch_image<T>(c, H, 0, s, 0, st, SpecParams{~0ull, 0.0f, 0.0f}))) return rc;
     } else if ((rc = launch_k1<T>(c, d, 0, s, b, 0, 0, 0, st))) {
         return rc;
     }
@@ -814,6 +866,10 @@ ss_status ss_create(int device, ss_context** out) {
     c->cfg.profile = 0;
     c->cfg.seed = 0x5A17;
     c->cfg.classify = 0;
+    c->cfg.fused_filter = 1;
+    c->cfg.spec_z = 4.0f;
+    c->cfg.spec_min_n = (int64_t)1 << 25;
+    c->cfg.spec_max_frac = 0.25f;
     DevGuard g(device);
     if (cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess) {
         (void)cudaGetLastError();
@@ -888,7 +944,18 @@ ss_status ss_set_config(ss_context* c, const ss_config* cfg) {
         return fail(c, SS_ERR_INVALID_ARGUMENT, "classify must be 0 (auto) or 1 (tree walk)");
     if (cfg->ctas_per_sm < 1 || cfg->ctas_per_sm > 16)
         return fail(c, SS_ERR_INVALID_ARGUMENT, "ctas_per_sm must be in [1, 16]");
-    const bool regrid = cfg->ctas_per_sm != c->cfg.ctas_per_sm || cfg->classify != c->cfg.classify;
+    if (cfg->fused_filter < 0 || cfg->fused_filter > 1)
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "fused_filter must be 0 or 1");
+    if (!(cfg->spec_z >= 0.0f && cfg->spec_z <= 64.0f))
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "spec_z must be in [0, 64]");
+    if (cfg->spec_min_n < 1)
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "spec_min_n must be >= 1");
+    if (!(cfg->spec_max_frac > 0.0f && cfg->spec_max_frac <= 1.0f))
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "spec_max_frac must be in (0, 1]");
+    // captured graphs bake in grid sizes and the fused-filter parameters
+    const bool regrid = cfg->ctas_per_sm != c->cfg.ctas_per_sm || cfg->classify != c->cfg.classify ||
+                        cfg->fused_filter != c->cfg.fused_filter || cfg->spec_z != c->cfg.spec_z ||
+                        cfg->spec_min_n != c->cfg.spec_min_n || cfg->spec_max_frac != c->cfg.spec_max_frac;
     c->cfg = *cfg;
     if (regrid)                   // captured grid sizes are stale (the other knobs are part of the graph key)
         for (auto& e : c->graphs) {

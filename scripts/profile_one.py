@@ -9,7 +9,8 @@ mode = sys.argv[2] if len(sys.argv) > 2 else "exact"
 b = int(sys.argv[3]) if len(sys.argv) > 3 else (256 if mode == "exact" else 1024)
 n = 1 << log2n
 x = torch.from_numpy(datagen.uniform(n, np.float32, seed=datagen.dataset_seed(5, 0))).cuda()
-ctx = ss.Context(0)
+import json
+ctx = ss.Context(0, **json.loads(os.environ.get('SS_CFG', '{}')))
 for _ in range(3):
     if mode == "exact":
         ctx.configure(b_exact=b); v = ctx.select(x, n // 2)

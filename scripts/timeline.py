@@ -12,7 +12,8 @@ mode = sys.argv[3] if len(sys.argv) > 3 else "exact"
 bd = int(sys.argv[4]) if len(sys.argv) > 4 else 0
 n = 1 << log2n
 x = torch.from_numpy(datagen.uniform(n, np.float32, seed=datagen.dataset_seed(5, 0))).cuda()
-ctx = ss.Context(0)
+import json
+ctx = ss.Context(0, **json.loads(os.environ.get('SS_CFG', '{}')))
 if mode == "exact":
     ctx.configure(b_exact=b, b_deep=bd)
 run = (lambda: ctx.select(x, n // 2)) if mode == "exact" else (lambda: ctx.approx_select(x, n // 2, b))
