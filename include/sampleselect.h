@@ -80,8 +80,9 @@ typedef struct {
                              miss falls back to a re-classifying filter); 0 = always the
                              paper's oracle bytes + filter kernel (§IV.B-c).  Same answer. */
     float spec_z;         /* window half-width in standard deviations of the sample rank of k
-                             (Binomial(s, k/n)); default 4 (miss probability ~6e-5) */
-    int64_t spec_min_n;   /* levels with at least this many elements speculate. default 2^25 */
+                             (Binomial(s, k/n)); default 3 (miss probability ~3e-3; a miss
+                             re-runs the level with the paper's filter) */
+    int64_t spec_min_n;   /* levels with at least this many elements speculate. default 2^22 */
     float spec_max_frac;  /* speculate only if the window holds at most this fraction of the
                              sample. default 0.25 */
     int32_t reserved_;

@@ -67,17 +67,16 @@ struct LevelCtl {
     u32 bucket;     // bucket j chosen at level l
     u32 ncta;       // active CTAs of the count/filter grid
     u32 marker;     // whole buckets inside the cell LUT's marker cells (tree_image_kernel)
-    // fused speculative filter: tree_image_kernel sets spec and
-    // the bucket window [wlo, whi] predicted from the sample; the count kernel
-    // then copies every element of the window to the next level's buffer
-    // (cap counts them) instead of writing oracle bytes, and its tail sets hit
-    // when the bucket holding k lies inside the window
+    // fused speculative filter (window_kernel): spec is set when
+    // the level streams once against the sample-predicted key window
+    // [klo, klo + kspan), copying it to the next level's buffer (cap counts
+    // it); hit = rank k fell inside the window
     u32 spec;
-    u32 wlo, whi;
     u32 hit;
     u64 cap;
     u64 klo, kspan; // the window as a key range: klo <= key < klo + kspan (mod 2^bits)
     u64 below;      // elements with key < klo (count kernel CTAs add theirs)
+    u64 wtot;       // elements inside the window (cap also counts the chunk padding)
     u32 nospec;     // set by a miss: this level re-runs the paper's filter on the same data
     u32 spec_eq;    // the window is one equality bucket (§IV.C): a hit returns its value
 };

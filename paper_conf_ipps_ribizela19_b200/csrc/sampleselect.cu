@@ -235,7 +235,7 @@ ss_status launch_count(ss_context* c, int H, const T* in, CountArgs& a, cudaStre
 // fused-filter count kernel: one CTA per SM, KW_STASH bytes of stash
 template <typename T>
 ss_status launch_window(ss_context* c, int /*H*/, const T* in, CountArgs a, cudaStream_t st) {
-    a.grid = (u32)c->sms;
+    a.grid = (u32)c->sms * (u32)KW_MINB;
     static bool attr_set[64] = {};
     if (!attr_set[c->device & 63]) {
         CK(cudaFuncSetAttribute(window_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)KW_STASH));
@@ -392,8 +392,9 @@ void prof_collect(ss_context* c) {
     (void)cudaGetLastError();
 }
 
-SpecParams spec_params(const ss_context* c) {
-    SpecParams p;
+struct SpecCfg { u64 min_n; float z, max_frac; };
+SpecCfg spec_params(const ss_context* c) {
+    SpecCfg p;
     p.min_n = c->cfg.fused_filter ? (u64)c->cfg.spec_min_n : ~0ull;
     p.z = c->cfg.spec_z;
     p.max_frac = c->cfg.spec_max_frac;
@@ -405,18 +406,19 @@ int expected_levels(const ss_context* c, u64 n, int b0, int bd, int s0, int sd, 
     // for s/b = 16); plan with 1.5x slack, fall back to more levels if needed.
     // A fused-filter level keeps its window: at most (2 (z sigma + 2) + 1) / s
     // of the level with sigma <= sqrt(s) / 2, plus one bucket at each end.
-    const SpecParams sp = spec_params(c);
+    const SpecCfg sp = spec_params(c);
     int L = 0;
     double m = (double)n;
     while (m > (double)B && L < SS_MAX_LEVELS - 2) {
-        const int b = L ? bd : b0, s = L ? sd : s0;
-        const double f = (2.0 * (sp.z * 0.5 * std::sqrt((double)s) + 2.0) + 1.0) / s;
-        const bool spec = s <= WIDE_K1_MAX_S && m >= (double)sp.min_n && f <= sp.max_frac;
         // levels whose size may reach min_n get the fused-filter kernel
-        // enqueued (it exits unless the device-side window decision is "spec")
-        if (spec_plan) spec_plan[L] = s <= WIDE_K1_MAX_S && f <= sp.max_frac && 2.0 * m >= (double)sp.min_n &&
-                                      sp.min_n != ~0ull;
-        m = spec ? m * 1.2 * (f + 2.0 / b) : m * 1.5 / b;
+        // enqueued (it exits unless the device-side window decision is
+        // "spec") and draw the level-0 sample size s0 (a narrower window)
+        const bool cand = s0 <= WIDE_K1_MAX_S && 2.0 * m >= (double)sp.min_n && sp.min_n != ~0ull;
+        const int b = L ? bd : b0, s = L && !cand ? sd : s0;
+        const double f = (2.0 * (sp.z * 0.5 * std::sqrt((double)s) + 2.0) + 1.0) / s;
+        const bool spec = cand && m >= (double)sp.min_n && f <= sp.max_frac;
+        if (spec_plan) spec_plan[L] = cand && f <= sp.max_frac;
+        m = spec ? m * 1.2 * f : m * 1.5 / b;
         ++L;
     }
     return L;
@@ -458,7 +460,7 @@ ss_status launch_k1_wide(ss_context* c, const T* in, int lev, int s, u32 B, cuda
 
 // K1b: the level's tree + count-kernel image from the wide K1's sorted sample.
 template <typename T>
-ss_status launch_image(ss_context* c, int H, int lev, int s, int fixup, cudaStream_t st, SpecParams sp) {
+ss_status launch_image(ss_context* c, int H, int lev, int s, int fixup, cudaStream_t st) {
     typedef typename Traits<T>::Key K;
     const K* sorted = reinterpret_cast<const K*>(c->d_sorted) + (size_t)lev * MAX_S;
     uint8_t* image = c->d_image + (size_t)lev * K2_IMAGE_SLOT;
@@ -469,7 +471,7 @@ ss_status launch_image(ss_context* c, int H, int lev, int s, int fixup, cudaStre
 #define SS_IMG_CASE(h)                                                                                     \
     case h:                                                                                                \
         CK(launch_pdl(tree_image_kernel<T, h>, dim3(IMG_CTAS), dim3(1024), 0, st, sorted, s, fixup, lut_on, \
-                      c->d_ctl + lev, c->d_res, image, tree, spl, eq, sp));                                \
+                      c->d_ctl + lev, c->d_res, image, tree, spl, eq));                                    \
         break;
     switch (H) {
         SS_IMG_CASE(2) SS_IMG_CASE(3) SS_IMG_CASE(4) SS_IMG_CASE(5) SS_IMG_CASE(6)
@@ -526,16 +528,8 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
         for (; lev < L; ++lev) {
             const int b = lev ? bd : b0, H = log2i(b);
             const u32 grid = grid_for<T>(c, H);
-            const int sl = lev ? s_deep : s;
+            const int sl = lev && !spec_plan[lev] ? s_deep : s;
             const bool wide = sl <= WIDE_K1_MAX_S;
-            if (wide) {
-                if ((rc2 = launch_k1_wide<T>(c, in, lev, sl, B, q, lev == 0 ? sample0 : nullptr))) return rc2;
-                if ((rc2 = launch_image<T>(c, H, lev, sl, 1, q,
-                                           spec_plan[lev] ? spec_params(c) : SpecParams{~0ull, 0.0f, 0.0f})))
-                    return rc2;
-            } else if ((rc2 = launch_k1<T>(c, in, lev, sl, b, 1, B, 0, q))) {
-                return rc2;
-            }
             CountArgs a{};
             if (wide) a.image = c->d_image + (size_t)lev * K2_IMAGE_SLOT;
             a.ctl = c->d_ctl + lev;
@@ -552,11 +546,25 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             a.level = lev;
             a.tail = TAIL_EXACT;
             a.cap_out = c->d_buf[lev & 1];   // the fused filter's window copy = next level's input
-            mark(c, lev, 1, 0, q);
-            if (wide && spec_plan[lev]) {             // fused filter (runs iff the window speculates)
-                if ((rc2 = launch_window<T>(c, H, in, a, q))) return rc2;
-                ++c->launches;
+            if (wide) {
+                if ((rc2 = launch_k1_wide<T>(c, in, lev, sl, B, q, lev == 0 ? sample0 : nullptr))) return rc2;
+                if (spec_plan[lev]) {         // fused filter (streams iff the sample window speculates)
+                    CountArgs w = a;
+                    const SpecCfg sp = spec_params(c);
+                    w.sorted = reinterpret_cast<K*>(c->d_sorted) + (size_t)lev * MAX_S;
+                    w.s = sl;
+                    w.spec_min_n = sp.min_n;
+                    w.spec_z = sp.z;
+                    w.spec_max_frac = sp.max_frac;
+                    mark(c, lev, 1, 0, q);
+                    if ((rc2 = launch_window<T>(c, H, in, w, q))) return rc2;
+                    ++c->launches;
+                }
+                if ((rc2 = launch_image<T>(c, H, lev, sl, 1, q))) return rc2;
+            } else if ((rc2 = launch_k1<T>(c, in, lev, sl, b, 1, B, 0, q))) {
+                return rc2;
             }
+            if (!(wide && spec_plan[lev])) mark(c, lev, 1, 0, q);
             if ((rc2 = launch_count<T>(c, H, in, a, q))) return rc2;
             mark(c, lev, 1, 1, q);
             ++c->launches;
@@ -754,7 +762,7 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     ++c->launches;
     if (wide) {
         if ((rc = launch_k1_wide<T>(c, d, 0, s, 0, st, sample0))) return rc;
-        if ((rc = launch_image<T>(c, H, 0, s, 0, st, SpecParams{~0ull, 0.0f, 0.0f}))) return rc;
+        if ((rc = launch_image<T>(c, H, 0, s, 0, st))) return rc;
     } else if ((rc = launch_k1<T>(c, d, 0, s, b, 0, 0, 0, st))) {
         return rc;
     }
@@ -867,8 +875,8 @@ ss_status ss_create(int device, ss_context** out) {
     c->cfg.seed = 0x5A17;
     c->cfg.classify = 0;
     c->cfg.fused_filter = 1;
-    c->cfg.spec_z = 4.0f;
-    c->cfg.spec_min_n = (int64_t)1 << 25;
+    c->cfg.spec_z = 3.0f;
+    c->cfg.spec_min_n = (int64_t)1 << 22;
     c->cfg.spec_max_frac = 0.25f;
     DevGuard g(device);
     if (cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess) {
