@@ -323,10 +323,22 @@ def run_ours(args, rank, world, local_rank):
     if rank != 0:
         return 0
 
-    # ---- roofline of the dominant kernel (K2, level 0: classify+count+oracle write)
+    # ---- roofline of the dominant kernel (level 0's count pass).  Exact
+    # selection at this size runs the fused filter on level 0 (window_kernel:
+    # reads the level once, writes the window = the next level); otherwise
+    # the paper's count kernel (reads the level, writes one oracle byte per
+    # element when exact).  Bytes per launch: DESIGN.md §7.
     peak, peak_src = measured_peak()
     S = np.dtype(args.dtype).itemsize
-    k2_bytes = (S + (1 if exact else 0)) * n          # read S*n, write n oracle bytes
+    fused0 = exact and bool(last.get("fused_levels", 0) & 1)
+    if fused0:
+        kname = "window_kernel (fused count + filter, level 0)"
+        k2_bytes = S * n + S * int(last["n_level"][1])
+        tkey = f"window_{args.mode}_{args.dtype}_2p{args.log2n}"
+    else:
+        kname = "count_kernel (K2, level 0)"
+        k2_bytes = (S + (1 if exact else 0)) * n          # read S*n, write n oracle bytes
+        tkey = f"count_{args.mode}_{args.dtype}_2p{args.log2n}"
     k2_avg = kavg(0, 1, prof_timed)
     achieved = k2_bytes / (k2_avg * 1e-3) / 1e9
     traffic = None
@@ -334,8 +346,7 @@ def run_ours(args, rank, world, local_rank):
     if os.path.exists(tpath):
         try:
             with open(tpath) as f:
-                tk = json.load(f).get(f"count_{args.mode}_{args.dtype}_2p{args.log2n}")
-            traffic = tk
+                traffic = json.load(f).get(tkey)
         except Exception:
             traffic = None
     path_bytes = float(last["bytes_algorithmic"])
@@ -347,13 +358,13 @@ def run_ours(args, rank, world, local_rank):
                                f"k=N/2, b={b}",
                    "n_per_gpu": n, "k": k, "b": b, "kind": args.kind,
                    "l2": "inputs larger than L2 (1 GiB input vs 126 MB L2); no flush"},
-        "roofline": {"bound": "hbm", "kernel": "count_kernel (K2, level 0)", "achieved": achieved,
+        "roofline": {"bound": "hbm", "kernel": kname, "achieved": achieved,
                      "peak": peak, "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
                      "peak_source": peak_src, "algorithmic_bytes": k2_bytes, "avg_ms": k2_avg,
                      "share_of_step": k2_avg / ms,
-                     "events": ("CUDA events around K2 on the call's stream, inside the timed loop"
+                     "events": ("CUDA events around the kernel on the call's stream, inside the timed loop"
                                 if args.events == "timed" else
-                                f"CUDA events around K2 on the call's stream, over a second timed pass of "
+                                f"CUDA events around the kernel on the call's stream, over a second timed pass of "
                                 f"{args.steps} steps right after the headline loop (events between the "
                                 f"kernels would break their PDL overlap in the headline loop)")},
         "path_roofline": {"algorithmic_bytes_per_step": path_bytes,

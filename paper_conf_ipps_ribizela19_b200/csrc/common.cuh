@@ -79,6 +79,8 @@ struct LevelCtl {
     u64 wtot;       // elements inside the window (cap also counts the chunk padding)
     u32 nospec;     // set by a miss: this level re-runs the paper's filter on the same data
     u32 spec_eq;    // the window is one equality bucket (§IV.C): a hit returns its value
+    u32 pre;        // this level's sample keys were gathered ahead (init / previous level's tail)
+    u32 pad2_;
 };
 
 struct SelectResult {

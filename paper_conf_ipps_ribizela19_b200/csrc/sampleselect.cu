@@ -9,6 +9,7 @@
 // case (rare: an unlucky sample) more levels are enqueued.  One device->host
 // copy per call returns the answer; there is no per-level host round trip.
 #include <algorithm>
+#include <chrono>
 #include <cmath>
 #include <atomic>
 #include <cstddef>
@@ -47,6 +48,7 @@ struct ss_context {
     uint8_t* d_eq = nullptr;     // [SS_MAX_LEVELS][MAX_B]
     u64* d_sorted = nullptr;     // [SS_MAX_LEVELS][MAX_S] sorted sample keys (wide K1)
     u64* d_sample0 = nullptr;    // [MAX_S] level-0 sample keys (gathered by the init kernel)
+    u64* d_presample = nullptr;  // [SS_MAX_LEVELS][MAX_S] sample keys gathered by a fused level's tail
     uint8_t* d_image = nullptr;  // [SS_MAX_LEVELS][K2_IMAGE_SLOT] count-kernel images (tree_image_kernel)
     SelectResult* h_res = nullptr;   // mapped pinned mirror of d_res (written by publish_kernel)
     SelectResult* h_res_dev = nullptr;
@@ -91,7 +93,14 @@ struct ss_context {
     long long calls_total = 0;
     int launches = 0;
     int64_t h2d = 0, d2h = 0;   // bytes copied by the current call
+    // SS_HOST_TIMING=1: host-side phase times of run_exact, printed by ss_destroy
+    bool host_timing = false;
+    double ht[5] = {};
+    long long ht_n = 0;
 };
+static inline double now_us() {
+    return std::chrono::duration<double, std::micro>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
 
 static constexpr u32 MAX_GRID = 2048;
 // SS_CARVEOUT (build flag): force one shared-memory carveout on every kernel
@@ -300,6 +309,7 @@ ss_status ensure_small(ss_context* c) {
     CK(cudaMalloc(&c->d_eq, (size_t)SS_MAX_LEVELS * MAX_B));
     CK(cudaMalloc(&c->d_sorted, sizeof(u64) * SS_MAX_LEVELS * MAX_S));
     CK(cudaMalloc(&c->d_sample0, sizeof(u64) * MAX_S));
+    CK(cudaMalloc(&c->d_presample, sizeof(u64) * SS_MAX_LEVELS * MAX_S));
     CK(cudaMalloc(&c->d_image, K2_IMAGE_SLOT * SS_MAX_LEVELS));
     CK(cudaHostAlloc(&c->h_res, sizeof(SelectResult), cudaHostAllocMapped));
     std::memset(c->h_res, 0, sizeof(SelectResult));
@@ -487,6 +497,7 @@ ss_status launch_image(ss_context* c, int H, int lev, int s, int fixup, cudaStre
 template <typename T>
 ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cudaStream_t st) {
     typedef typename Traits<T>::Key K;
+    const double t_in = c->host_timing ? now_us() : 0.0;
     // reading R7: level 0 draws s = clamp(16 b, 4096, 16384) samples (or the
     // configured size); deeper levels hold n_l ~ n / b elements and draw
     // S_DEEP = max(1024, b) -- a quarter of the sort, ~1.25x the bucket size
@@ -529,6 +540,13 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             const int b = lev ? bd : b0, H = log2i(b);
             const u32 grid = grid_for<T>(c, H);
             const int sl = lev && !spec_plan[lev] ? s_deep : s;
+            const int sl_next = lev + 1 < L && !spec_plan[lev + 1] ? s_deep : s;
+            K* pre_next = lev + 1 < L && sl_next <= WIDE_K1_MAX_S
+                              ? reinterpret_cast<K*>(c->d_presample) + (size_t)(lev + 1) * MAX_S : nullptr;
+            const void* pre_this = lev == 0 ? (const void*)sample0
+                                            : (spec_plan[lev - 1] ? (const void*)(reinterpret_cast<K*>(c->d_presample) +
+                                                                                  (size_t)lev * MAX_S)
+                                                                  : nullptr);
             const bool wide = sl <= WIDE_K1_MAX_S;
             CountArgs a{};
             if (wide) a.image = c->d_image + (size_t)lev * K2_IMAGE_SLOT;
@@ -547,7 +565,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             a.tail = TAIL_EXACT;
             a.cap_out = c->d_buf[lev & 1];   // the fused filter's window copy = next level's input
             if (wide) {
-                if ((rc2 = launch_k1_wide<T>(c, in, lev, sl, B, q, lev == 0 ? sample0 : nullptr))) return rc2;
+                if ((rc2 = launch_k1_wide<T>(c, in, lev, sl, B, q, pre_this))) return rc2;
                 if (spec_plan[lev]) {         // fused filter (streams iff the sample window speculates)
                     CountArgs w = a;
                     const SpecCfg sp = spec_params(c);
@@ -556,17 +574,32 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
                     w.spec_min_n = sp.min_n;
                     w.spec_z = sp.z;
                     w.spec_max_frac = sp.max_frac;
+                    w.sample_next = pre_next;
+                    w.s_next = sl_next;
+                    w.seed = (u64)c->cfg.seed;
                     mark(c, lev, 1, 0, q);
                     if ((rc2 = launch_window<T>(c, H, in, w, q))) return rc2;
+                    mark(c, lev, 1, 1, q);        // slot (lev, K2) = the fused kernel on planned levels
                     ++c->launches;
                 }
-                if ((rc2 = launch_image<T>(c, H, lev, sl, 1, q))) return rc2;
+                if (lev == 0 || spec_plan[lev]) {
+                    if ((rc2 = launch_image<T>(c, H, lev, sl, 1, q))) return rc2;
+                } else {
+                    // small deeper level: each count CTA builds the tree from
+                    // the sorted sample itself and walks it (no image kernel,
+                    // no lookup table)
+                    a.image = nullptr;
+                    a.sorted = reinterpret_cast<K*>(c->d_sorted) + (size_t)lev * MAX_S;
+                    a.s = sl;
+                    a.fixup = 1;
+                    a.lut = 0;
+                }
             } else if ((rc2 = launch_k1<T>(c, in, lev, sl, b, 1, B, 0, q))) {
                 return rc2;
             }
             if (!(wide && spec_plan[lev])) mark(c, lev, 1, 0, q);
             if ((rc2 = launch_count<T>(c, H, in, a, q))) return rc2;
-            mark(c, lev, 1, 1, q);
+            if (!(wide && spec_plan[lev])) mark(c, lev, 1, 1, q);
             ++c->launches;
             if (a.grid != grid) return fail(c, SS_ERR_INTERNAL, "grid mismatch");
             T* out = reinterpret_cast<T*>(c->d_buf[lev & 1]);
@@ -680,14 +713,20 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             CK(cudaGraphExecKernelNodeSetParams(ge->exec, ge->init_node, &ge->init_params));
         }
         ge->stamp = ++c->graph_clock;
+        if (c->host_timing) c->ht[0] += now_us() - t_in;
+        const double t_l = c->host_timing ? now_us() : 0.0;
         CK(cudaGraphLaunch(ge->exec, st));
+        if (c->host_timing) c->ht[1] += now_us() - t_l;
         c->launches += ge->kernels;
     } else {
         if ((rc = enqueue_init(st))) return rc;
         if ((rc = enqueue_levels(0, st))) return rc;
         if ((rc = enqueue_publish(c, st))) return rc;
     }
+    const double t_w = c->host_timing ? now_us() : 0.0;
     if ((rc = wait_publish(c, st))) return rc;
+    if (c->host_timing) c->ht[2] += now_us() - t_w;
+    const double t_s = c->host_timing ? now_us() : 0.0;
     // rare: an unlucky sample left more than B elements after the planned levels
     while (!c->h_res->done) {
         if (!c->h_res->incomplete || L >= SS_MAX_LEVELS - 2)
@@ -739,6 +778,11 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     c->launches_total += c->launches;
     c->calls_total += 1;
     prof_collect(c);
+    if (c->host_timing) {
+        c->ht[3] += now_us() - t_s;
+        c->ht[4] += now_us() - t_in;
+        ++c->ht_n;
+    }
     return SS_OK;
 }
 
@@ -866,6 +910,7 @@ ss_status ss_create(int device, ss_context** out) {
     ss_context* c = new (std::nothrow) ss_context();
     if (!c) return SS_ERR_OUT_OF_MEMORY;
     c->device = device;
+    c->host_timing = std::getenv("SS_HOST_TIMING") != nullptr;
     c->cfg.b_exact = 256;
     c->cfg.b_deep = 0;
     c->cfg.sample_size = 0;
@@ -899,6 +944,10 @@ ss_status ss_create(int device, ss_context** out) {
 
 void ss_destroy(ss_context* c) {
     if (!c) return;
+    if (c->host_timing && c->ht_n)
+        std::fprintf(stderr, "ss host timing (us/call over %lld exact calls): prep %.2f graph-launch %.2f "
+                     "wait %.2f post %.2f total %.2f\n", c->ht_n, c->ht[0] / c->ht_n, c->ht[1] / c->ht_n,
+                     c->ht[2] / c->ht_n, c->ht[3] / c->ht_n, c->ht[4] / c->ht_n);
     DevGuard g(c->device);
     cudaFree(c->d_oracles);
     cudaFree(c->d_buf[0]);
@@ -913,6 +962,7 @@ void ss_destroy(ss_context* c) {
     cudaFree(c->d_eq);
     cudaFree(c->d_sorted);
     cudaFree(c->d_sample0);
+    cudaFree(c->d_presample);
     cudaFree(c->d_image);
     cudaFree(c->d_seq);
     for (auto& e : c->graphs) {

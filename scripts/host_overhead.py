@@ -20,3 +20,6 @@ print(f"ctx._stream(None): {t(lambda: ctx._stream(None)):.2f} us")
 print(f"select n=1000: {t(lambda: ctx.select(x, 500), 500):.2f} us")
 xs = torch.rand(1 << 16, device="cuda")
 print(f"select n=2^16: {t(lambda: ctx.select(xs, 1 << 15), 500):.2f} us")
+xb = torch.rand(1 << 28, device="cuda")
+print(f"select n=2^28: {t(lambda: ctx.select(xb, 1 << 27), 50):.2f} us")
+ctx.close()
