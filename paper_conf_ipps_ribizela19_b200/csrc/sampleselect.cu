@@ -242,15 +242,16 @@ ss_status launch_count(ss_context* c, int H, const T* in, CountArgs& a, cudaStre
 }
 
 // fused-filter count kernel: one CTA per SM, KW_STASH bytes of stash
-template <typename T>
+template <typename T, bool APX = false>
 ss_status launch_window(ss_context* c, int /*H*/, const T* in, CountArgs a, cudaStream_t st) {
     a.grid = (u32)c->sms * (u32)KW_MINB;
     static bool attr_set[64] = {};
     if (!attr_set[c->device & 63]) {
-        CK(cudaFuncSetAttribute(window_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)KW_STASH));
+        CK(cudaFuncSetAttribute(window_kernel<T, APX>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                (int)KW_STASH));
         attr_set[c->device & 63] = true;
     }
-    CK(launch_pdl(window_kernel<T>, dim3(a.grid), dim3(KW_THREADS), KW_STASH, st, in, a));
+    CK(launch_pdl(window_kernel<T, APX>, dim3(a.grid), dim3(KW_THREADS), KW_STASH, st, in, a));
     CKLAUNCH("window_kernel");
     return SS_OK;
 }
@@ -436,7 +437,7 @@ int expected_levels(const ss_context* c, u64 n, int b0, int bd, int s0, int sd, 
 
 template <typename T>
 ss_status launch_k1(ss_context* c, const T* in, int lev, int s, int b, int fixup, u32 B, int final_level,
-                    cudaStream_t st) {
+                    cudaStream_t st, void* sorted_out = nullptr) {
     typedef typename Traits<T>::Key K;
     K* tree = reinterpret_cast<K*>(c->d_tree) + (size_t)lev * MAX_B;
     K* spl = reinterpret_cast<K*>(c->d_spl) + (size_t)lev * MAX_B;
@@ -444,7 +445,7 @@ ss_status launch_k1(ss_context* c, const T* in, int lev, int s, int b, int fixup
     mark(c, lev, 0, 0, st);
     CK(launch_pdl(sample_tree_kernel<T>, dim3(1), dim3(K1_THREADS), k1_smem<T>(s, B), st,
                   in, c->d_ctl + lev, c->d_res, tree, spl, eq, s, b, fixup, B, (u64)c->cfg.seed, lev,
-                  final_level));
+                  final_level, reinterpret_cast<K*>(sorted_out)));
     CKLAUNCH("sample_tree_kernel");
     mark(c, lev, 0, 1, st);
     ++c->launches;
@@ -804,10 +805,14 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
                   (int)MAX_B, c->d_res, n, k, (int)(c->cfg.profile == 3), d, s, (u64)c->cfg.seed, sample0));
     CKLAUNCH("init_kernel");
     ++c->launches;
+    // fused one-pass window (approx_window in kernels.cuh) on large inputs;
+    // the paper's full count runs only if it cannot decide
+    const SpecCfg sp = spec_params(c);
+    const bool fw = sp.min_n != ~0ull && n >= sp.min_n;
+    K* sorted0 = reinterpret_cast<K*>(c->d_sorted);
     if (wide) {
         if ((rc = launch_k1_wide<T>(c, d, 0, s, 0, st, sample0))) return rc;
-        if ((rc = launch_image<T>(c, H, 0, s, 0, st))) return rc;
-    } else if ((rc = launch_k1<T>(c, d, 0, s, b, 0, 0, 0, st))) {
+    } else if ((rc = launch_k1<T>(c, d, 0, s, b, 0, 0, 0, st, fw ? sorted0 : nullptr))) {
         return rc;
     }
     CountArgs a{};
@@ -826,8 +831,21 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     a.level = 0;
     a.tail = TAIL_APPROX;
     mark(c, 0, 1, 0, st);
+    if (fw) {
+        CountArgs w = a;
+        w.sorted = sorted0;
+        w.s = s;
+        w.b = b;
+        w.spec_min_n = sp.min_n;
+        w.spec_z = sp.z;
+        w.spec_max_frac = 1.0f;
+        if ((rc = launch_window<T, true>(c, H, d, w, st))) return rc;
+        mark(c, 0, 1, 1, st);
+        ++c->launches;
+    }
+    if (wide && (rc = launch_image<T>(c, H, 0, s, 0, st))) return rc;
     if ((rc = launch_count<T>(c, H, d, a, st))) return rc;
-    mark(c, 0, 1, 1, st);
+    if (!fw) mark(c, 0, 1, 1, st);
     ++c->launches;
     if ((rc = enqueue_publish(c, st))) return rc;
     if ((rc = wait_publish(c, st))) return rc;
@@ -838,6 +856,8 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     ss_stats& S = c->stats;
     std::memset(&S, 0, sizeof(S));
     S.levels = 1;
+    S.spec_levels = (int32_t)r.spec_levels;
+    S.fused_levels = (int32_t)r.fused_levels;
     S.lut_ctas = (int32_t)r.lut_stats[0];
     S.lut_marker = (int32_t)r.lut_stats[1];
     S.n_level[0] = (int64_t)n;

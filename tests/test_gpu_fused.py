@@ -135,3 +135,44 @@ def test_fused_default_large(cuda_device):
         assert st["spec_levels"] & 1 and st["fused_levels"] & 1, st
         assert st["bytes_algorithmic"] < 5.0 * n
     c.close()
+
+
+# ------------------------------------------------- approximate variant -----
+@pytest.mark.parametrize("dtype", DTYPES)
+@pytest.mark.parametrize("b", [64, 256, 1024])
+@pytest.mark.parametrize("z", [3.0, 0.0])
+def test_fused_approx_matches_mirror(cuda_device, dtype, b, z):
+    """§II.C through the one-pass splitter window (approx_window): the same
+    splitter and the exact rank as the oracle's mirror with the same seed,
+    whether the window decides (z = 3) or mostly falls back (z = 0)."""
+    import paper_conf_ipps_ribizela19_b200 as ss
+    c = ss.Context(0, spec_min_n=1, spec_z=z)
+    n = (1 << 20) + 5
+    x = _gen("normal", n, dtype, seed=b + 1)
+    xd = _dev(x)
+    s = oracle.sample_size(b)
+    seed = c.config["seed"]
+    decided = 0
+    for k in _ranks(n, b):
+        v, r = c.approx_select(xd, k, b)
+        vo, ro, _ = oracle.approx_select(x, k, b, s, seed)
+        assert _bits(v) == _bits(vo) and r == ro, (k, v, vo, r, ro)
+        decided += c.stats()["fused_levels"] & 1
+    if z == 3.0:
+        assert decided >= 5, decided
+    c.close()
+
+
+def test_fused_approx_duplicates(cuda_device):
+    import paper_conf_ipps_ribizela19_b200 as ss
+    c = ss.Context(0, spec_min_n=1)
+    for kind in ("distinct16", "distinct1024", "equal"):
+        n = (1 << 20) + 1
+        x = _gen(kind, n, np.float32, seed=4)
+        xd = _dev(x)
+        for k in _ranks(n, 2):
+            for b in (64, 1024):
+                v, r = c.approx_select(xd, k, b)
+                vo, ro, _ = oracle.approx_select(x, k, b, oracle.sample_size(b), c.config["seed"])
+                assert _bits(v) == _bits(vo) and r == ro, (kind, k, b)
+    c.close()
