@@ -288,6 +288,10 @@ ss_status set_k1_attrs(ss_context* c) {
     CK(cudaFuncSetAttribute(filter_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)FILTER_SMEM));
     CK(cudaFuncSetAttribute(sample_rank_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                             (int)(16384 * sizeof(K))));
+    CK(cudaFuncSetAttribute(sample_chunk_sort_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)(K1C_CHUNK * sizeof(K))));
+    CK(cudaFuncSetAttribute(sample_merge_rank_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)(16384 * sizeof(K))));
     // one carveout (all shared) for every kernel of the path: no L1/shared
     // reconfiguration between consecutive kernels
 #ifdef SS_CARVEOUT
@@ -799,9 +803,10 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     if (c->cfg.profile && (rc = prof_init(c))) return rc;
     c->launches = 0;
     c->d2h = 0;
-    const bool wide = s <= WIDE_K1_MAX_S;
-    K* sample0 = wide ? reinterpret_cast<K*>(c->d_sample0) : nullptr;
-    CK(launch_pdl(init_kernel<T>, dim3(wide ? (u32)s / 256u : 1u), dim3(256), 0, st, c->d_ctl, 2, c->d_totals,
+    const bool merge = s > WIDE_K1_MAX_S && s % (int)K1C_CHUNK == 0;   // chunk sort + merge rank
+    const bool wide = s <= WIDE_K1_MAX_S || merge;
+    K* sample0 = s <= WIDE_K1_MAX_S ? reinterpret_cast<K*>(c->d_sample0) : nullptr;
+    CK(launch_pdl(init_kernel<T>, dim3(sample0 ? (u32)s / 256u : 1u), dim3(256), 0, st, c->d_ctl, 2, c->d_totals,
                   (int)MAX_B, c->d_res, n, k, (int)(c->cfg.profile == 3), d, s, (u64)c->cfg.seed, sample0));
     CKLAUNCH("init_kernel");
     ++c->launches;
@@ -810,7 +815,18 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     const SpecCfg sp = spec_params(c);
     const bool fw = sp.min_n != ~0ull && n >= sp.min_n;
     K* sorted0 = reinterpret_cast<K*>(c->d_sorted);
-    if (wide) {
+    if (merge) {
+        K* chunks = reinterpret_cast<K*>(c->d_sorted) + MAX_S;   // level 1's slot: scratch here
+        mark(c, 0, 0, 0, st);
+        CK(launch_pdl(sample_chunk_sort_kernel<T>, dim3((u32)s / K1C_CHUNK), dim3(1024), K1C_CHUNK * sizeof(K), st,
+                      d, c->d_ctl, c->d_res, chunks, (u64)c->cfg.seed, 0));
+        CKLAUNCH("sample_chunk_sort_kernel");
+        CK(launch_pdl(sample_merge_rank_kernel<T>, dim3((u32)s / 1024u), dim3(1024), (size_t)s * sizeof(K), st,
+                      c->d_ctl, c->d_res, chunks, s, sorted0, 0));
+        CKLAUNCH("sample_merge_rank_kernel");
+        mark(c, 0, 0, 1, st);
+        c->launches += 2;
+    } else if (wide) {
         if ((rc = launch_k1_wide<T>(c, d, 0, s, 0, st, sample0))) return rc;
     } else if ((rc = launch_k1<T>(c, d, 0, s, b, 0, 0, 0, st, fw ? sorted0 : nullptr))) {
         return rc;
