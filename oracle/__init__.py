@@ -70,6 +70,9 @@ def _load():
             lib.oracle_filter_bucket.argtypes = [i32, vp, i64, vp, i32, vp]
             lib.oracle_filter_bucket.restype = i64
             lib.oracle_approx_select.argtypes = [i32, vp, i64, i64, i32, i64, u64, vp, p64, p64]
+            lib.oracle_select_upper.argtypes = [i32, vp, i64, i64, vp]
+            lib.oracle_select_upper_bruteforce.argtypes = [i32, vp, i64, i64, vp]
+            lib.oracle_select_upper_bruteforce.restype = i64
             lib.oracle_sampleselect.argtypes = [i32, vp, i64, i64, i32, i64, i64, u64, vp, p64, i32]
             _lib = lib
     return _lib
@@ -116,6 +119,31 @@ def select_bruteforce(data, k: int):
     if rc:
         raise ValueError("oracle_select_bruteforce: invalid argument")
     return out[0]
+
+
+def select_upper(data, k: int) -> np.ndarray:
+    """§IV.I L606-615 (top-k fusion): the kth-smallest element and all larger
+    elements = positions k..n-1 of the sorted sequence (ascending)."""
+    a = _arr(data)
+    if not 0 <= k < a.size:
+        raise ValueError(f"oracle_select_upper: invalid argument (n={a.size}, k={k})")
+    out = np.empty(a.size - int(k), dtype=a.dtype)
+    rc = _load().oracle_select_upper(DTYPES[a.dtype], _ptr(a), a.size, int(k), _ptr(out))
+    if rc:
+        raise ValueError(f"oracle_select_upper: rc={rc}")
+    return out
+
+
+def select_upper_bruteforce(data, k: int) -> np.ndarray:
+    """O(n^2) count definition of :func:`select_upper` (unordered multiset)."""
+    a = _arr(data)
+    if not 0 <= k < a.size:
+        raise ValueError("oracle_select_upper_bruteforce: invalid argument")
+    out = np.empty(a.size - int(k), dtype=a.dtype)
+    w = _load().oracle_select_upper_bruteforce(DTYPES[a.dtype], _ptr(a), a.size, int(k), _ptr(out))
+    if w != a.size - int(k):
+        raise ValueError(f"oracle_select_upper_bruteforce: wrote {w} of {a.size - int(k)}")
+    return out
 
 
 def count_less(data, v) -> int:

@@ -35,6 +35,12 @@
  *   oracle_filter_bucket        extract one bucket, input order     (§IV.B-c)
  *   oracle_approx_select        approximate selection: splitter whose rank
  *                               r_i is closest to k (§II.C, §V.G)
+ *   oracle_select_upper         top-k fusion: the kth-smallest element and
+ *                               "all larger elements" = positions k..n-1 of
+ *                               the sorted sequence (§IV.I, reading R22)
+ *   oracle_select_upper_bruteforce
+ *                               O(n^2): value v appears #{x<=v} - max(#{x<v}, k)
+ *                               times among ranks >= k (§IV.I, §II)
  *
  * Parity pins (tests/test_oracle.py, -m "not gpu"): hand-worked examples
  * (tests/golden/), min/max special cases, numpy.partition on NaN-free data,
@@ -143,6 +149,44 @@ int oracle_select_bruteforce(int dt, const void* data, int64_t n, int64_t k, voi
         if (lt <= k && k < le) { memcpy(out, v, S); return OR_OK; }
     }
     return OR_EINVAL; /* unreachable for a valid k */
+}
+
+/* §IV.I: "not only the kth-smallest element is required, but also
+ * all larger elements" -- positions k..n-1 of the sorted sequence, written to
+ * out[0..n-k) in ascending order. */
+int oracle_select_upper(int dt, const void* data, int64_t n, int64_t k, void* out) {
+    size_t S = elem_size(dt);
+    if (!S || !data || !out || n < 1 || k < 0 || k >= n) return OR_EINVAL;
+    char* buf = (char*)malloc((size_t)n * S);
+    if (!buf) return OR_ENOMEM;
+    memcpy(buf, data, (size_t)n * S);
+    sort_copy(dt, buf, n);
+    memcpy(out, buf + (size_t)k * S, (size_t)(n - k) * S);
+    free(buf);
+    return OR_OK;
+}
+
+/* The same multiset by counting, O(n^2): the copies of a value v occupy the
+ * ranks #{x<v} .. #{x<=v}-1 (L86-88), so #{x<=v} - max(#{x<v}, k) of them (if
+ * positive) have rank >= k.  Each distinct value (first occurrence) is emitted
+ * that many times, in input order of first occurrence.  Returns the count. */
+int64_t oracle_select_upper_bruteforce(int dt, const void* data, int64_t n, int64_t k, void* out) {
+    size_t S = elem_size(dt);
+    if (!S || !data || !out || n < 1 || k < 0 || k >= n) return -1;
+    const char* p = (const char*)data;
+    char* o = (char*)out;
+    int64_t w = 0;
+    for (int64_t i = 0; i < n; ++i) {
+        const void* v = p + (size_t)i * S;
+        int seen = 0;
+        for (int64_t j = 0; j < i && !seen; ++j) seen = oracle_cmp(dt, p + (size_t)j * S, v) == 0;
+        if (seen) continue;
+        int64_t lt = oracle_count_less(dt, data, n, v);
+        int64_t le = oracle_count_leq(dt, data, n, v);
+        int64_t m = le - (lt > k ? lt : k);
+        for (int64_t c = 0; c < m; ++c) memcpy(o + (size_t)(w++) * S, v, S);
+    }
+    return w;
 }
 
 /* ---------------------------------------------------------------------------

@@ -333,3 +333,62 @@ def test_approx_error_statistics(b):
     errs = np.array(errs)
     assert 0.4 / (4 * b) <= errs.mean() <= 2.5 / (4 * b)
     assert errs.max() <= 4.0 / b
+
+
+# ------------------------------------------- top-k fusion (§IV.I) ------------
+def _sorted_bits(a):
+    a = np.asarray(a)
+    u = np.uint32 if a.dtype.itemsize == 4 else np.uint64
+    return sorted(int(v) for v in a.view(u))
+
+
+@pytest.mark.parametrize("case", _load("upper_examples.json")["cases"], ids=lambda c: c["cite"][:40])
+def test_golden_select_upper(case):
+    dt = np.dtype(case["dtype"])
+    if "bits" in case:
+        x = _bits_array(case["bits"], dt)
+        exp = [int(b, 16) for b in case["expect_bits"]]
+        got = oracle.select_upper(x, case["k"])
+        assert [_bits(v) for v in got] == exp
+        assert _sorted_bits(oracle.select_upper_bruteforce(x, case["k"])) == sorted(exp)
+    else:
+        x = np.array(case["values"], dtype=dt)
+        assert oracle.select_upper(x, case["k"]).tolist() == case["expect"]
+        assert sorted(oracle.select_upper_bruteforce(x, case["k"]).tolist()) == case["expect"]
+
+
+@settings(max_examples=150, deadline=None)
+@given(st.lists(_f32_special, min_size=1, max_size=40), st.data())
+def test_select_upper_bruteforce_tiny_special_f32(bits, data):
+    x = np.array(bits, dtype=np.uint32).view(np.float32)
+    k = data.draw(st.integers(0, len(bits) - 1))
+    up = oracle.select_upper(x, k)
+    assert up.size == len(bits) - k
+    assert _sorted_bits(up) == _sorted_bits(oracle.select_upper_bruteforce(x, k))
+    pos = {int(b, 16): i for i, b in enumerate(F32_ORDER)}
+    if all(b in pos for b in bits):   # independent: the hand-ordered totalOrder table
+        assert [_bits(v) for v in up] == sorted(bits, key=lambda b: pos[b])[k:]
+
+
+@settings(max_examples=150, deadline=None)
+@given(st.lists(st.integers(-3, 3), min_size=1, max_size=50), st.data())
+def test_select_upper_bruteforce_tiny_duplicates_int64(vals, data):
+    x = np.array(vals, dtype=np.int64)
+    k = data.draw(st.integers(0, len(vals) - 1))
+    assert oracle.select_upper(x, k).tolist() == sorted(vals)[k:]
+    assert sorted(oracle.select_upper_bruteforce(x, k).tolist()) == sorted(vals)[k:]
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64, np.int32, np.int64])
+def test_select_upper_special_cases_and_numpy(dtype):
+    """k = 0 -> the input as a multiset; k = n-1 -> [max]; NaN-free data with
+    no mixed +-0 -> numpy.sort(x)[k:] (library special case); the first output
+    is select(x, k) (the definition of §IV.I)."""
+    x = datagen.make("normal" if np.dtype(dtype).kind == "f" else "int", 3001, dtype, seed=11)
+    x = x[x != 0] if np.dtype(dtype).kind == "f" else x
+    assert _sorted_bits(oracle.select_upper(x, 0)) == _sorted_bits(x)
+    assert oracle.select_upper(x, x.size - 1).tolist() == [np.max(x)]
+    for k in (1, x.size // 3, x.size - 2):
+        up = oracle.select_upper(x, k)
+        assert np.array_equal(up, np.sort(x)[k:])
+        assert _bits(up[0]) == _bits(oracle.select(x, k))
