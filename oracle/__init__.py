@@ -71,6 +71,7 @@ def _load():
             lib.oracle_filter_bucket.restype = i64
             lib.oracle_approx_select.argtypes = [i32, vp, i64, i64, i32, i64, u64, vp, p64, p64]
             lib.oracle_select_upper.argtypes = [i32, vp, i64, i64, vp]
+            lib.oracle_select_multi.argtypes = [i32, vp, i64, i32, p64, vp]
             lib.oracle_select_upper_bruteforce.argtypes = [i32, vp, i64, i64, vp]
             lib.oracle_select_upper_bruteforce.restype = i64
             lib.oracle_sampleselect.argtypes = [i32, vp, i64, i64, i32, i64, i64, u64, vp, p64, i32]
@@ -131,6 +132,19 @@ def select_upper(data, k: int) -> np.ndarray:
     rc = _load().oracle_select_upper(DTYPES[a.dtype], _ptr(a), a.size, int(k), _ptr(out))
     if rc:
         raise ValueError(f"oracle_select_upper: rc={rc}")
+    return out
+
+
+def select_multi(data, ks) -> np.ndarray:
+    """Reading R23: the elements of ranks ks (0-based, §II
+    L82-88 per rank) -- one sort, m indexings."""
+    a = _arr(data)
+    k = np.ascontiguousarray(np.asarray(ks, dtype=np.int64).reshape(-1))
+    out = np.empty(k.size, dtype=a.dtype)
+    rc = _load().oracle_select_multi(DTYPES[a.dtype], _ptr(a), a.size, int(k.size),
+                                     k.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)), _ptr(out))
+    if rc:
+        raise ValueError(f"oracle_select_multi: invalid argument (n={a.size}, ks={k.tolist()[:8]})")
     return out
 
 

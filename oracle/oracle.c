@@ -38,6 +38,8 @@
  *   oracle_select_upper         top-k fusion: the kth-smallest element and
  *                               "all larger elements" = positions k..n-1 of
  *                               the sorted sequence (§IV.I, reading R22)
+ *   oracle_select_multi         m ranks: the elements at positions k_1..k_m of
+ *                               the sorted sequence (reading R23)
  *   oracle_select_upper_bruteforce
  *                               O(n^2): value v appears #{x<=v} - max(#{x<v}, k)
  *                               times among ranks >= k (§IV.I, §II)
@@ -162,6 +164,22 @@ int oracle_select_upper(int dt, const void* data, int64_t n, int64_t k, void* ou
     memcpy(buf, data, (size_t)n * S);
     sort_copy(dt, buf, n);
     memcpy(out, buf + (size_t)k * S, (size_t)(n - k) * S);
+    free(buf);
+    return OR_OK;
+}
+
+/* Reading R23 (§VI): m ranks -- the definition of
+ * §II L82-88 applied to each k_i; one sort, m indexings. */
+int oracle_select_multi(int dt, const void* data, int64_t n, int32_t m, const int64_t* ks, void* out) {
+    size_t S = elem_size(dt);
+    if (!S || !data || !out || !ks || n < 1 || m < 1) return OR_EINVAL;
+    for (int32_t i = 0; i < m; ++i)
+        if (ks[i] < 0 || ks[i] >= n) return OR_EINVAL;
+    char* buf = (char*)malloc((size_t)n * S);
+    if (!buf) return OR_ENOMEM;
+    memcpy(buf, data, (size_t)n * S);
+    sort_copy(dt, buf, n);
+    for (int32_t i = 0; i < m; ++i) memcpy((char*)out + (size_t)i * S, buf + (size_t)ks[i] * S, S);
     free(buf);
     return OR_OK;
 }

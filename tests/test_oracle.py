@@ -392,3 +392,31 @@ def test_select_upper_special_cases_and_numpy(dtype):
         up = oracle.select_upper(x, k)
         assert np.array_equal(up, np.sort(x)[k:])
         assert _bits(up[0]) == _bits(oracle.select(x, k))
+
+
+# ------------------------------------- multi-rank selection (NEXT-2) ---------
+@settings(max_examples=100, deadline=None)
+@given(st.lists(st.integers(-3, 3), min_size=1, max_size=40), st.data())
+def test_select_multi_bruteforce_tiny(vals, data):
+    """Each rank against the O(n^2) count definition and Python's sort."""
+    x = np.array(vals, dtype=np.int64)
+    ks = data.draw(st.lists(st.integers(0, len(vals) - 1), min_size=1, max_size=8))
+    got = oracle.select_multi(x, ks)
+    assert got.tolist() == [sorted(vals)[k] for k in ks]
+    assert got.tolist() == [int(oracle.select_bruteforce(x, k)) for k in ks]
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64, np.int32, np.int64])
+def test_select_multi_monotone_and_numpy(dtype):
+    """Ranks in increasing order give non-decreasing results (totalOrder);
+    NaN-free data without mixed +-0 equals numpy.sort indexing; repeats and
+    the extremes are allowed."""
+    x = datagen.make("normal" if np.dtype(dtype).kind == "f" else "int", 5003, dtype, seed=17)
+    x = x[x != 0] if np.dtype(dtype).kind == "f" else x
+    ks = [0, 1, 7, 7, x.size // 2, x.size - 1]
+    got = oracle.select_multi(x, ks)
+    assert np.array_equal(got, np.sort(x)[ks])
+    for a, b in zip(got[:-1], got[1:]):
+        assert oracle.cmp(a, b, dtype) <= 0
+    with pytest.raises(ValueError):
+        oracle.select_multi(x, [x.size])
