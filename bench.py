@@ -43,7 +43,10 @@ def parse():
     p.add_argument("--log2n", type=int, default=28, help="elements per GPU = 2^log2n")
     p.add_argument("--dtype", default="float32", choices=["float32", "float64", "int32", "int64"])
     p.add_argument("--kind", default="uniform")
-    p.add_argument("--mode", default="exact", choices=["exact", "approx"])
+    p.add_argument("--mode", default="exact", choices=["exact", "approx", "upper", "multi"],
+                   help="upper: top-k fusion (select + all larger elements, §IV.I), k = n - --upper-count")
+    p.add_argument("--upper-count", type=int, default=1 << 20, help="upper mode: n - k elements returned")
+    p.add_argument("--ranks", type=int, default=8, help="multi mode: number of ranks (seeded, uniform)")
     p.add_argument("--b", type=int, default=0, help="buckets (exact default 256, approx 1024)")
     p.add_argument("--e2e-steps", type=int, default=0, help="host-buffer steps (default: min(steps, 10))")
     p.add_argument("--cpu-seconds", type=float, default=10.0, help="CPU-oracle baseline budget")
@@ -172,12 +175,14 @@ def run_reference(args, rank, world):
     oracle.build()
     m = min(x.size, 1 << 22)
     sample = np.ascontiguousarray(x[:m])
-    kind = "exact" if args.mode == "exact" else "approx"
+    kind = args.mode
     b = args.b or (256 if kind == "exact" else 1024)
 
     def step():
         if kind == "exact":
             oracle.select(sample, m // 2)
+        elif kind == "upper":
+            oracle.select_upper(sample, m - min(args.upper_count, m))
         else:
             oracle.approx_select(sample, m // 2, b, oracle.sample_size(b), 0x5A17)
     for _ in range(args.warmup):
@@ -195,7 +200,7 @@ def run_reference(args, rank, world):
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": _dt_name(args.dtype),
         "data": "synthetic", "config": cfg,
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": 1, "kind": "oracle",
-                         "sample": f"oracle {'select' if kind == 'exact' else 'approx_select'} "
+                         "sample": f"oracle {dict(exact='select', upper='select_upper').get(kind, 'approx_select')} "
                                    f"(CPU, 1 thread) on the first {m} elements of the workload per step"},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
@@ -222,7 +227,9 @@ def run_ours(args, rank, world, local_rank):
     ctx = ss.Context(dev)
     if args.classify:
         ctx.configure(classify=args.classify)
-    exact = args.mode == "exact"
+    upper = args.mode == "upper"
+    multi = args.mode == "multi"
+    exact = args.mode in ("exact", "upper", "multi")
     b = args.b or (256 if exact else 1024)
     if exact:
         ctx.configure(b_exact=b)
@@ -234,6 +241,18 @@ def run_ours(args, rank, world, local_rank):
 
         def step(inp):
             return sel.select(inp, k)
+    elif multi:
+        ks = np.random.default_rng(12345).integers(0, n, args.ranks).tolist()
+        k = ks[0]
+
+        def step(inp):
+            return ctx.select_multi(inp, ks)
+    elif upper:
+        k = n - args.upper_count
+        outbuf = torch.empty(args.upper_count, dtype=xd.dtype, device=xd.device)
+
+        def step(inp):
+            return ctx.select_upper(inp, k, out=outbuf)
     else:
         k = n // 2
         if exact:
@@ -272,10 +291,13 @@ def run_ours(args, rank, world, local_rank):
     barrier()
     ms = ev0.elapsed_time(ev1) / args.steps
     prof_timed = ctx.profile_totals(reset=True)
+    upper_ms = []
     if args.events == "separate":
         ctx.configure(profile=2)
         for _ in range(args.steps):
             step(xd)
+            if upper:
+                upper_ms.append(ctx.stats()["ms_upper_gather"])
         torch.cuda.synchronize()
         prof_timed = ctx.profile_totals(reset=True)
     # per-kernel breakdown (all kernels timed; separate, informational pass)
@@ -301,7 +323,7 @@ def run_ours(args, rank, world, local_rank):
     # ---- end-to-end through the public API with HOST buffers
     e2e_steps = args.e2e_steps or min(args.steps, 10)
     xhn = xh.numpy()
-    if world == 1:
+    if world == 1 and not upper and not multi:
         step_h = (lambda: ctx.select(xhn, k)) if exact else (lambda: ctx.approx_select(xhn, k, b))
         step_h()
         torch.cuda.synchronize()
@@ -331,7 +353,15 @@ def run_ours(args, rank, world, local_rank):
     peak, peak_src = measured_peak()
     S = np.dtype(args.dtype).itemsize
     fused0 = exact and bool(last.get("fused_levels", 0) & 1)
-    if fused0:
+    if multi:
+        kname = "whole call (shared sample + count, bucket extractions, per-rank tails)"
+        k2_bytes = float(last["bytes_algorithmic"])
+        tkey = f"multi_{args.dtype}_2p{args.log2n}"
+    elif upper:
+        kname = "upper_gather_kernel (top-k pass: read the input, write the elements > result)"
+        k2_bytes = S * n + S * int(last["upper_greater"])
+        tkey = f"upper_{args.dtype}_2p{args.log2n}"
+    elif fused0:
         kname = "window_kernel (fused count + filter, level 0)"
         k2_bytes = S * n + S * int(last["n_level"][1])
         tkey = f"window_{args.mode}_{args.dtype}_2p{args.log2n}"
@@ -339,7 +369,7 @@ def run_ours(args, rank, world, local_rank):
         kname = "count_kernel (K2, level 0)"
         k2_bytes = (S + (1 if exact else 0)) * n          # read S*n, write n oracle bytes
         tkey = f"count_{args.mode}_{args.dtype}_2p{args.log2n}"
-    k2_avg = kavg(0, 1, prof_timed)
+    k2_avg = float(np.mean(upper_ms)) if upper and upper_ms else (ms if multi else kavg(0, 1, prof_timed))
     achieved = k2_bytes / (k2_avg * 1e-3) / 1e9
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -355,7 +385,8 @@ def run_ours(args, rank, world, local_rank):
         "warmup": max(3, args.warmup), "ms_per_step": ms, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": _dt_name(args.dtype), "data": "synthetic",
         "config": {"workload": f"{args.mode} select n=2^{args.log2n} {args.dtype} {args.kind} per GPU, "
-                               f"k=N/2, b={b}",
+                               + (f"k=N-{args.upper_count} (+ all larger elements), b={b}" if upper else
+                                  f"{args.ranks} seeded uniform ranks in one call, b={b}" if multi else f"k=N/2, b={b}"),
                    "n_per_gpu": n, "k": k, "b": b, "kind": args.kind,
                    "l2": "inputs larger than L2 (1 GiB input vs 126 MB L2); no flush"},
         "roofline": {"bound": "hbm", "kernel": kname, "achieved": achieved,

@@ -37,7 +37,7 @@
 extern "C" {
 #endif
 
-#define SS_ABI_VERSION 3
+#define SS_ABI_VERSION 4
 #define SS_MAX_LEVELS 32
 
 typedef enum { SS_FLOAT32 = 0, SS_FLOAT64 = 1, SS_INT32 = 2, SS_INT64 = 3 } ss_dtype;
@@ -113,6 +113,11 @@ typedef struct {
     int32_t fused_levels;              /* bit l: ... and its window held bucket j (hit: the
                                           captured window is level l+1; else the fallback
                                           filter re-read level l) */
+    int64_t upper_greater;             /* ss_select_upper: #{x > result} (the rest of the
+                                          output is copies of result) */
+    float ms_upper_gather;             /* ss_select_upper with profile != 0: device ms of the
+                                          upper_gather_kernel pass (CUDA events) */
+    int32_t reserved_stats_;
 } ss_stats;
 
 /* ---- context --------------------------------------------------------- */
@@ -153,6 +158,28 @@ ss_status ss_approx_select(ss_context* ctx, ss_dtype dt, const void* d_data, int
 ss_status ss_approx_select_host(ss_context* ctx, ss_dtype dt, const void* h_data, int64_t n,
                                 int64_t k, int32_t b, void* h_result, int64_t* h_rank, void* stream);
 
+/* ---- selection with all larger elements: top-k fusion (§IV.I) ----
+ * "not only the kth-smallest element is required, but also all larger
+ * elements": writes the element of rank k to *h_result (as ss_select) and the
+ * n-k elements of ranks k..n-1 (IEEE totalOrder / numeric order, reading R3)
+ * to d_out[0..n-k), a caller-owned DEVICE buffer of at least n-k elements of
+ * dtype dt that must not overlap d_data.  The output is a multiset: its order
+ * is unspecified (elements > result first, then n-k-#{x > result} copies of
+ * result; reading R22).  Errors as ss_select; d_out == NULL is
+ * SS_ERR_INVALID_ARGUMENT.  Synchronises `stream`. */
+ss_status ss_select_upper(ss_context* ctx, ss_dtype dt, const void* d_data, int64_t n, int64_t k,
+                          void* d_out, void* h_result, void* stream);
+
+/* ---- multi-rank selection (§VI; reading R23) ------
+ * Writes the element of rank h_ks[i] to h_results[i] (m elements of dtype dt,
+ * host memory) for i < m, 1 <= m <= 1024, every h_ks[i] in [0, n) (any order,
+ * repeats allowed).  For n >= 2^20 and m >= 4 the ranks share one sample, one splitter
+ * tree and one count pass; each distinct bucket holding a rank is extracted
+ * once and finished by the single-rank path.  Results are bit-identical to m
+ * calls of ss_select.  d_data: device, naturally aligned.  Synchronises. */
+ss_status ss_select_multi(ss_context* ctx, ss_dtype dt, const void* d_data, int64_t n, int32_t m,
+                          const int64_t* h_ks, void* h_results, void* stream);
+
 /* ---- single steps of one level (per-kernel parity tests, sharded driver) --
  * All are asynchronous on `stream` and touch only the buffers passed in.  Keys
  * are the order-preserving unsigned images of the values (u32 for 4-byte,
@@ -185,6 +212,24 @@ ss_status ss_step_count(ss_context* ctx, ss_dtype dt, const void* d_data, int64_
 ss_status ss_step_filter(ss_context* ctx, ss_dtype dt, const void* d_data, int64_t n,
                          const uint8_t* d_oracles, int32_t bucket, void* d_out, uint64_t* d_count,
                          void* stream);
+
+/* Atomics ablation (§V.E, Fig. 6, Fig. 8
+ * right L1093-1120): the same per-bucket totals as ss_step_count (d_totals[b]
+ * uint64, overwritten; no oracle bytes) from a plain Fig. 4 count kernel whose
+ * bucket increments are applied by `mode`:
+ *   0 SS_ABL_SHARED      shared-memory atomics
+ *   1 SS_ABL_SHARED_WA   shared, warp-aggregated (__match_any_sync)
+ *   2 SS_ABL_SHARED_FIG6 shared, warp-aggregated by Fig. 6's per-bit ballots (reading R13)
+ *   3 SS_ABL_GLOBAL      global atomics on d_totals
+ *   4 SS_ABL_GLOBAL_WA   global, warp-aggregated
+ * b: power of two in [2, 1024]; tree as for ss_step_count.  Not used by
+ * ss_select (the product's count kernel has its own histogram);
+ * it exists to measure the paper's design space on B200. */
+enum { SS_ABL_SHARED = 0, SS_ABL_SHARED_WA = 1, SS_ABL_SHARED_FIG6 = 2, SS_ABL_GLOBAL = 3,
+       SS_ABL_GLOBAL_WA = 4 };
+ss_status ss_step_count_ablation(ss_context* ctx, ss_dtype dt, const void* d_data, int64_t n,
+                                 const void* d_tree, int32_t b, int32_t mode, uint64_t* d_totals,
+                                 void* stream);
 
 /* ---- sharded (multi-GPU) selection support -------------------
  * The sharded driver (paper_conf_ipps_ribizela19_b200/sharded.py) runs one

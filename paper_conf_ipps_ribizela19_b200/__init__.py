@@ -104,7 +104,8 @@ class Context:
                 "ms_kernel": [list(s.ms_kernel[l]) for l in range(L + 1)],
                 "tl_us": [[list(s.tl_us[l][q]) for q in range(3)] for l in range(L + 1)],
                 "spec_levels": s.spec_levels, "fused_levels": s.fused_levels,
-                "lut_ctas": s.lut_ctas}
+                "lut_ctas": s.lut_ctas, "upper_greater": s.upper_greater,
+                "ms_upper_gather": s.ms_upper_gather}
 
     def raw_tl(self):
         """profile=3: the full 32x3 timeline (us after init; -1 = not stamped)."""
@@ -163,6 +164,37 @@ class Context:
                        ctypes.byref(rank), self._stream(stream)))
         return out[0], int(rank.value)
 
+    def select_upper(self, x, k: int, out=None, stream=None):
+        """Top-k fusion (§IV.I): the element of rank k and the n-k
+        elements of ranks k..n-1 (a multiset, order unspecified).  x must be a
+        CUDA tensor; returns (value, out) with out a tensor of n-k elements."""
+        if not _is_tensor(x):
+            raise TypeError("select_upper takes a CUDA tensor (the output is a device buffer)")
+        dt, p, n, npdt, dev = self._args(x)
+        if out is None:
+            import torch
+            out = torch.empty(max(n - int(k), 0), dtype=x.dtype, device=x.device)
+        elif out.dtype != x.dtype or out.device != x.device or not out.is_contiguous() or \
+                out.numel() < n - int(k):
+            raise ValueError("out must be a contiguous tensor of x's dtype/device with >= n-k elements")
+        val = np.empty(1, dtype=npdt)
+        self._check(self._lib.ss_select_upper(self._h, dt, p, n, int(k), ctypes.c_void_p(out.data_ptr()),
+                                              ctypes.c_void_p(val.ctypes.data), self._stream(stream)))
+        return val[0], out
+
+    def select_multi(self, x, ks, stream=None):
+        """Multi-rank selection: the elements of ranks ks
+        (0-based) of the CUDA tensor x, as a numpy array; one shared count pass."""
+        if not _is_tensor(x):
+            raise TypeError("select_multi takes a CUDA tensor")
+        dt, p, n, npdt, _ = self._args(x)
+        ka = np.ascontiguousarray(np.asarray(ks, dtype=np.int64).reshape(-1))
+        out = np.empty(ka.size, dtype=npdt)
+        self._check(self._lib.ss_select_multi(self._h, dt, p, n, int(ka.size),
+                                              ka.ctypes.data_as(ctypes.POINTER(ctypes.c_int64)),
+                                              ctypes.c_void_p(out.ctypes.data), self._stream(stream)))
+        return out
+
     # -------------------------------------------- single steps (tensors) --
     def step_sample(self, x, level: int, slot_begin: int, count: int, out_keys, stream=None):
         dt, p, n, _, _ = self._args(x)
@@ -182,6 +214,15 @@ class Context:
                                             ctypes.c_void_p(totals.data_ptr()),
                                             ctypes.c_void_p(oracles.data_ptr() if oracles is not None else 0),
                                             self._stream(stream)))
+
+    def step_count_ablation(self, x, tree, b: int, mode, totals, stream=None):
+        """Atomics ablation: bucket totals from the plain
+        Fig. 4 count kernel with the increment strategy `mode` (a name from
+        _abi.ABLATION_MODES or its code)."""
+        dt, p, n, _, _ = self._args(x)
+        m = _abi.ABLATION_MODES[mode] if isinstance(mode, str) else int(mode)
+        self._check(self._lib.ss_step_count_ablation(self._h, dt, p, n, ctypes.c_void_p(tree.data_ptr()), int(b), m,
+                                                     ctypes.c_void_p(totals.data_ptr()), self._stream(stream)))
 
     def step_filter(self, x, oracles, bucket: int, out, count, stream=None):
         dt, p, n, _, _ = self._args(x)
@@ -230,3 +271,13 @@ def select(x, k: int):
 def approx_select(x, k: int, b: int = 1024):
     """(approximate value, its exact rank) with b buckets, one level."""
     return default_context(_device_of(x)).approx_select(x, k, b)
+
+
+def select_upper(x, k: int, out=None):
+    """(element of rank k, tensor of the n-k elements of rank >= k) -- top-k, §IV.I."""
+    return default_context(_device_of(x)).select_upper(x, k, out)
+
+
+def select_multi(x, ks):
+    """Elements of ranks ks of x (one shared sample + count pass)."""
+    return default_context(_device_of(x)).select_multi(x, ks)

@@ -14,6 +14,7 @@ LIB_PATH = os.environ.get("SS_LIB") or os.path.join(_PKG, "libsampleselect.so")
 
 SS_FLOAT32, SS_FLOAT64, SS_INT32, SS_INT64 = 0, 1, 2, 3
 SS_MAX_LEVELS = 32
+ABLATION_MODES = {"shared": 0, "shared_wa": 1, "shared_fig6": 2, "global": 3, "global_wa": 4}
 STATUS = {0: "SS_OK", 1: "SS_ERR_INVALID_ARGUMENT", 2: "SS_ERR_CUDA",
           3: "SS_ERR_OUT_OF_MEMORY", 5: "SS_ERR_INTERNAL"}
 
@@ -21,8 +22,8 @@ STATUS = {0: "SS_OK", 1: "SS_ERR_INVALID_ARGUMENT", 2: "SS_ERR_CUDA",
 EXPORTS = [
     "ss_create", "ss_destroy", "ss_get_config", "ss_set_config", "ss_last_stats", "ss_profile_totals",
     "ss_last_error", "ss_status_string", "ss_abi_version",
-    "ss_select", "ss_select_host", "ss_approx_select", "ss_approx_select_host",
-    "ss_step_sample", "ss_step_tree", "ss_step_count", "ss_step_filter",
+    "ss_select", "ss_select_host", "ss_approx_select", "ss_approx_select_host", "ss_select_upper", "ss_select_multi",
+    "ss_step_sample", "ss_step_tree", "ss_step_count", "ss_step_count_ablation", "ss_step_filter",
     "ss_step_search", "ss_step_keys_to_values",
 ]
 
@@ -47,7 +48,9 @@ class SSStats(ctypes.Structure):
                 ("ms_kernel", (ctypes.c_float * 3) * SS_MAX_LEVELS),
                 ("tl_us", ((ctypes.c_float * 2) * 3) * SS_MAX_LEVELS),
                 ("lut_ctas", ctypes.c_int32), ("lut_marker", ctypes.c_int32),
-                ("spec_levels", ctypes.c_int32), ("fused_levels", ctypes.c_int32)]
+                ("spec_levels", ctypes.c_int32), ("fused_levels", ctypes.c_int32),
+                ("upper_greater", ctypes.c_int64), ("ms_upper_gather", ctypes.c_float),
+                ("reserved_stats_", ctypes.c_int32)]
 
 
 class SSError(RuntimeError):
@@ -91,9 +94,12 @@ def lib() -> ctypes.CDLL:
         L.ss_select_host.argtypes = [vp, st, vp, i64, i64, vp, vp]
         L.ss_approx_select.argtypes = [vp, st, vp, i64, i64, i32, vp, ctypes.POINTER(i64), vp]
         L.ss_approx_select_host.argtypes = [vp, st, vp, i64, i64, i32, vp, ctypes.POINTER(i64), vp]
+        L.ss_select_upper.argtypes = [vp, st, vp, i64, i64, vp, vp, vp]
+        L.ss_select_multi.argtypes = [vp, st, vp, i64, i32, ctypes.POINTER(i64), vp, vp]
         L.ss_step_sample.argtypes = [vp, st, vp, i64, i32, i64, i64, vp, vp]
         L.ss_step_tree.argtypes = [vp, st, vp, i32, i32, i32, vp, vp, vp, vp]
         L.ss_step_count.argtypes = [vp, st, vp, i64, vp, i32, vp, vp, vp]
+        L.ss_step_count_ablation.argtypes = [vp, st, vp, i64, vp, i32, i32, vp, vp]
         L.ss_step_filter.argtypes = [vp, st, vp, i64, vp, i32, vp, vp, vp]
         L.ss_step_search.argtypes = [vp, vp, i32, i64, vp, vp, vp]
         L.ss_step_keys_to_values.argtypes = [vp, st, vp, i64, vp, vp]

@@ -94,6 +94,14 @@ struct ss_context {
     int launches = 0;
     int64_t h2d = 0, d2h = 0;   // bytes copied by the current call
     // SS_HOST_TIMING=1: host-side phase times of run_exact, printed by ss_destroy
+    unsigned long long* d_upper_cnt = nullptr;  // ss_select_upper: #{x > result}
+    cudaEvent_t ev_upper[2] = {nullptr, nullptr};
+    unsigned upper_attr = 0;                    // bit dt_code: gather kernel smem attribute set
+    // ss_select_multi: scratch (sample keys, tree, splitters, eq, totals, search
+    // results, bucket counts, one value) and the extracted buckets
+    unsigned char* d_multi_scratch = nullptr;
+    void* d_multi = nullptr;
+    size_t cap_multi = 0;
     bool host_timing = false;
     double ht[5] = {};
     long long ht_n = 0;
@@ -888,6 +896,216 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     return SS_OK;
 }
 
+template <typename T>
+ss_status launch_ablation(ss_context* c, const T* d, u64 n, const void* tree, int h, int mode, u64* totals,
+                          cudaStream_t st) {
+    typedef typename Traits<T>::Key K;
+    const u32 grid = (u32)c->sms * 2;
+    const K* tr = (const K*)tree;
+    unsigned long long* tt = (unsigned long long*)totals;
+    switch (mode) {
+        case ABL_SHARED: ablation_count_kernel<T, ABL_SHARED><<<grid, ABL_THREADS, 0, st>>>(d, n, tr, h, tt); break;
+        case ABL_SHARED_WA: ablation_count_kernel<T, ABL_SHARED_WA><<<grid, ABL_THREADS, 0, st>>>(d, n, tr, h, tt); break;
+        case ABL_SHARED_FIG6: ablation_count_kernel<T, ABL_SHARED_FIG6><<<grid, ABL_THREADS, 0, st>>>(d, n, tr, h, tt); break;
+        case ABL_GLOBAL: ablation_count_kernel<T, ABL_GLOBAL><<<grid, ABL_THREADS, 0, st>>>(d, n, tr, h, tt); break;
+        default: ablation_count_kernel<T, ABL_GLOBAL_WA><<<grid, ABL_THREADS, 0, st>>>(d, n, tr, h, tt); break;
+    }
+    CK(cudaGetLastError());
+    c->launches_total += 1;
+    return SS_OK;
+}
+
+// Top-k fusion (§IV.I; reading R22): the exact select, then one
+// streaming pass that appends the elements > result to d_out, then the
+// copies of result that fill it up to n-k.
+template <typename T>
+ss_status run_upper(ss_context* c, const T* d, u64 n, u64 k, T* d_out, void* h_result, cudaStream_t st) {
+    typedef typename Traits<T>::Key K;
+    ss_status rc = run_exact<T>(c, d, n, k, h_result, st);
+    if (rc) return rc;
+    if (!c->d_upper_cnt) CK(cudaMalloc(&c->d_upper_cnt, sizeof(unsigned long long)));
+    const bool prof = c->cfg.profile != 0;
+    if (prof && !c->ev_upper[0]) {
+        CK(cudaEventCreate(&c->ev_upper[0]));
+        CK(cudaEventCreate(&c->ev_upper[1]));
+    }
+    T v;
+    std::memcpy(&v, h_result, sizeof(T));
+    K vb;
+    std::memcpy(&vb, &v, sizeof(T));
+    const K kv = Traits<T>::to_key(vb);
+    const u64 m = n - k;
+    CK(cudaMemsetAsync(c->d_upper_cnt, 0, sizeof(unsigned long long), st));
+    constexpr u64 EPV = 16 / sizeof(T);
+    const u64 tiles = (n / EPV + (u64)UG_THREADS * UG_VEC - 1) / ((u64)UG_THREADS * UG_VEC);
+    const u32 grid = (u32)std::max<u64>(1, std::min<u64>(tiles, (u64)c->sms * UG_MINB));
+    if (prof) CK(cudaEventRecord(c->ev_upper[0], st));
+    if (!(c->upper_attr >> dt_code<T>() & 1)) {   // stage > 48 KB-safe default: opt in once per (context device, dtype)
+        CK(cudaFuncSetAttribute(upper_gather_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, UG_STAGE_BYTES));
+        c->upper_attr |= 1u << dt_code<T>();
+    }
+    upper_gather_kernel<T><<<grid, UG_THREADS, UG_STAGE_BYTES, st>>>(d, n, kv, d_out, c->d_upper_cnt);
+    CK(cudaGetLastError());
+    if (prof) CK(cudaEventRecord(c->ev_upper[1], st));
+    upper_fill_kernel<T><<<(u32)c->sms * 4, 256, 0, st>>>(d_out, m, v, c->d_upper_cnt);
+    CK(cudaGetLastError());
+    unsigned long long greater = 0;
+    CK(cudaMemcpyAsync(&greater, c->d_upper_cnt, sizeof(greater), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    if (greater >= m && m > 0) return fail(c, SS_ERR_INTERNAL, "select_upper: #{x > result} >= n-k");
+    c->stats.upper_greater = (int64_t)greater;
+    c->stats.bytes_algorithmic += (double)sizeof(T) * ((double)n + (double)m);   // one read + the output
+    c->stats.launches += 2;
+    c->stats.d2h_bytes += (int64_t)sizeof(greater);
+    c->launches_total += 2;
+    if (prof) {
+        float ms = 0;
+        CK(cudaEventElapsedTime(&ms, c->ev_upper[0], c->ev_upper[1]));
+        c->stats.ms_upper_gather = ms;
+    }
+    return SS_OK;
+}
+
+// Multi-rank selection (§VI "multiple ... selection",
+// reading R23): m ranks share one sample, one splitter tree and ONE count
+// pass over the input (the dominant K2 pass, §IV.G); every distinct bucket
+// holding a rank is extracted once (K5, all extractions before any deeper
+// level because the deeper levels reuse the oracle bytes), and each rank then
+// finishes with the single-rank select on its bucket (rank k - r_j, Fig. 1).
+// An equality bucket answers its ranks with its splitter (§IV.C).
+constexpr int MULTI_MAX = 1024;
+constexpr u64 MULTI_MIN_N = (u64)1 << 20;   // below: one select per rank is cheaper
+// Below 4 ranks the per-rank fused selects win: measured at n = 2^28 fp32
+// (profiles/r01f_next_rows.md) the shared path costs ~0.50 ms + ~0.18 ms per
+// extra rank, a fused single select 0.28 ms.
+constexpr int MULTI_MIN_M = 4;
+
+template <typename T>
+ss_status run_multi(ss_context* c, ss_dtype dt, const T* d, u64 n, int m, const int64_t* ks, void* h_res,
+                    cudaStream_t st) {
+    typedef typename Traits<T>::Key K;
+    unsigned char* outb = (unsigned char*)h_res;
+    ss_status rc;
+    double bytes = 0;
+    int launches = 0;
+    if (n < MULTI_MIN_N || m < MULTI_MIN_M) {
+        for (int i = 0; i < m; ++i) {
+            if ((rc = run_exact<T>(c, d, n, (u64)ks[i], outb + (size_t)i * sizeof(T), st))) return rc;
+            bytes += c->stats.bytes_algorithmic;
+            launches += c->stats.launches;
+        }
+        c->stats.bytes_algorithmic = bytes;
+        c->stats.launches = launches;
+        return SS_OK;
+    }
+    const int b = std::min(c->cfg.b_exact, 256);
+    const int s = c->cfg.sample_size > 0 ? c->cfg.sample_size : sample_size(c->cfg, b);
+    // scratch layout (8-byte slots)
+    const size_t o_keys = 0, o_tree = o_keys + (size_t)MAX_S * 8, o_spl = o_tree + (size_t)MAX_B * 8,
+                 o_tot = o_spl + (size_t)MAX_B * 8, o_srch = o_tot + (size_t)MAX_B * 8,
+                 o_cnt = o_srch + (size_t)MULTI_MAX * 32, o_val = o_cnt + (size_t)MULTI_MAX * 8,
+                 o_eq = o_val + 64, o_lut = o_eq + MAX_B, o_sb = o_lut + 256,
+                 o_sbase = o_sb + (size_t)MF_MAX_SLOTS * 4, scratch = o_sbase + (size_t)MF_MAX_SLOTS * 8;
+    if (!c->d_multi_scratch) CK(cudaMalloc(&c->d_multi_scratch, scratch));
+    unsigned char* S0 = c->d_multi_scratch;
+    if ((rc = ensure_small(c))) return rc;
+    if ((rc = grow(c, (void**)&c->d_oracles, &c->cap_oracles, (size_t)n + 64))) return rc;
+    if ((rc = ss_step_sample(c, dt, d, (int64_t)n, 0, 0, s, S0 + o_keys, st))) return rc;
+    if ((rc = ss_step_tree(c, dt, S0 + o_keys, s, b, 1, S0 + o_tree, S0 + o_spl, S0 + o_eq, st))) return rc;
+    if ((rc = ss_step_count(c, dt, d, (int64_t)n, S0 + o_tree, b, (uint64_t*)(S0 + o_tot), c->d_oracles, st)))
+        return rc;
+    for (int i = 0; i < m; ++i)
+        if ((rc = ss_step_search(c, (const uint64_t*)(S0 + o_tot), b, ks[i], S0 + o_eq,
+                                 (int64_t*)(S0 + o_srch) + 4 * (size_t)i, st)))
+            return rc;
+    std::vector<int64_t> sr((size_t)m * 4);
+    CK(cudaMemcpyAsync(sr.data(), S0 + o_srch, sizeof(int64_t) * 4 * (size_t)m, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    int step_launches = 3 + m;
+    bytes += (double)sizeof(T) * n + (double)n;   // count: read + oracle bytes
+    // distinct buckets, in bucket order; regions of d_multi for the non-equality ones
+    std::vector<int> order(m);
+    for (int i = 0; i < m; ++i) order[i] = i;
+    std::sort(order.begin(), order.end(), [&](int a, int bb) { return sr[4 * (size_t)a] < sr[4 * (size_t)bb]; });
+    std::vector<int64_t> bucket_off(MAX_B, -1);
+    size_t total = 0;
+    for (int i : order) {
+        const int64_t j = sr[4 * (size_t)i], nj = sr[4 * (size_t)i + 2], eq = sr[4 * (size_t)i + 3];
+        if (eq || bucket_off[j] >= 0) continue;
+        bucket_off[j] = (int64_t)total;
+        total += (size_t)nj;
+    }
+    if ((rc = grow(c, &c->d_multi, &c->cap_multi, std::max<size_t>(total, 1) * sizeof(T)))) return rc;
+    std::vector<u32> slot_bucket;
+    std::vector<u64> slot_base;
+    for (int j = 0; j < b; ++j)
+        if (bucket_off[j] >= 0) {
+            slot_bucket.push_back((u32)j);
+            slot_base.push_back((u64)bucket_off[j]);
+        }
+    const int nb = (int)slot_bucket.size();
+    if (nb >= 2 && nb <= MF_MAX_SLOTS && b <= 256) {
+        // one pass over the oracle bytes extracts every wanted bucket
+        std::vector<uint8_t> slot_of(256, 0xFF);
+        for (int i = 0; i < nb; ++i) slot_of[slot_bucket[i]] = (uint8_t)i;
+        CK(cudaMemcpyAsync(S0 + o_lut, slot_of.data(), 256, cudaMemcpyHostToDevice, st));
+        CK(cudaMemcpyAsync(S0 + o_sb, slot_bucket.data(), sizeof(u32) * nb, cudaMemcpyHostToDevice, st));
+        CK(cudaMemcpyAsync(S0 + o_sbase, slot_base.data(), sizeof(u64) * nb, cudaMemcpyHostToDevice, st));
+        multi_filter_kernel<T><<<c->step_grid, MF_THREADS, 0, st>>>(
+            d, n, c->d_oracles, c->d_cta_counts, (u32)b, c->step_grid, S0 + o_lut, (const u32*)(S0 + o_sb),
+            (const u64*)(S0 + o_sbase), (u32)nb, (T*)c->d_multi);
+        CK(cudaGetLastError());
+        step_launches += 1;
+        bytes += (double)n;    // one read of the oracle bytes
+        CK(cudaStreamSynchronize(st));   // the host slot vectors go out of scope
+    } else {
+        for (int i = 0; i < nb; ++i) {
+            if ((rc = ss_step_filter(c, dt, d, (int64_t)n, c->d_oracles, (int32_t)slot_bucket[i],
+                                     (T*)c->d_multi + slot_base[i], (uint64_t*)(S0 + o_cnt) + i, st)))
+                return rc;
+            step_launches += 1;
+        }
+        bytes += (double)nb * n;   // each extraction reads the oracle bytes
+    }
+    for (int i = 0; i < m; ++i) {
+        const int64_t j = sr[4 * (size_t)i], kk = sr[4 * (size_t)i + 1], nj = sr[4 * (size_t)i + 2],
+                      eq = sr[4 * (size_t)i + 3];
+        if (!eq) bytes += 2.0 * sizeof(T) * nj;
+        (void)kk;
+    }
+    // equality buckets: the value is splitter j (1-based), keys -> values
+    for (int i = 0; i < m; ++i) {
+        const int64_t j = sr[4 * (size_t)i], eq = sr[4 * (size_t)i + 3];
+        if (!eq) continue;
+        if ((rc = ss_step_keys_to_values(c, dt, S0 + o_spl + (size_t)(j - 1) * sizeof(K), 1, S0 + o_val, st)))
+            return rc;
+        CK(cudaMemcpyAsync(outb + (size_t)i * sizeof(T), S0 + o_val, sizeof(T), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));   // S0 + o_val is reused by the next equality rank
+        step_launches += 1;
+    }
+    CK(cudaStreamSynchronize(st));
+    // the remaining levels of each rank: single-rank select on its bucket
+    for (int i = 0; i < m; ++i) {
+        const int64_t j = sr[4 * (size_t)i], kk = sr[4 * (size_t)i + 1], nj = sr[4 * (size_t)i + 2],
+                      eq = sr[4 * (size_t)i + 3];
+        if (eq) continue;
+        if ((rc = run_exact<T>(c, (const T*)c->d_multi + bucket_off[j], (u64)nj, (u64)kk,
+                               outb + (size_t)i * sizeof(T), st)))
+            return rc;
+        bytes += c->stats.bytes_algorithmic;
+        launches += c->stats.launches;
+    }
+    c->launches_total += step_launches;
+    std::memset(&c->stats, 0, sizeof(c->stats));
+    c->stats.levels = 1;
+    c->stats.n_level[0] = (int64_t)n;
+    c->stats.n_level[1] = (int64_t)total;
+    c->stats.bytes_algorithmic = bytes;
+    c->stats.launches = launches + step_launches;
+    c->stats.d2h_bytes = (int64_t)(sizeof(int64_t) * 4 * (size_t)m);
+    return SS_OK;
+}
+
 ss_status check_common(ss_context* c, ss_dtype dt, const void* p, int64_t n, int64_t k, void* out) {
     if (!c) return SS_ERR_INVALID_ARGUMENT;
     if (!dt_size(dt)) return fail(c, SS_ERR_INVALID_ARGUMENT, "unknown dtype");
@@ -1001,6 +1219,11 @@ void ss_destroy(ss_context* c) {
     cudaFree(c->d_presample);
     cudaFree(c->d_image);
     cudaFree(c->d_seq);
+    cudaFree(c->d_upper_cnt);
+    cudaFree(c->d_multi_scratch);
+    cudaFree(c->d_multi);
+    for (auto& e : c->ev_upper)
+        if (e) cudaEventDestroy(e);
     for (auto& e : c->graphs) {
         if (e.exec) cudaGraphExecDestroy(e.exec);
         if (e.graph) cudaGraphDestroy(e.graph);
@@ -1116,6 +1339,49 @@ ss_status ss_select_host(ss_context* c, ss_dtype dt, const void* h_data, int64_t
     cudaStream_t st = (cudaStream_t)stream;
     if ((rc = stage_host(c, h_data, (size_t)n * dt_size(dt), st))) return rc;
     return select_impl(c, dt, c->d_stage, n, k, h_result, stream);
+}
+
+ss_status ss_select_upper(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k, void* d_out,
+                          void* h_result, void* stream) {
+    ss_status rc = check_common(c, dt, d_data, n, k, h_result);
+    if (rc) return rc;
+    if (!d_out) return fail(c, SS_ERR_INVALID_ARGUMENT, "d_out is NULL");
+    const size_t S = dt_size(dt);
+    const uintptr_t a0 = (uintptr_t)d_data, a1 = a0 + (size_t)n * S, o0 = (uintptr_t)d_out,
+                    o1 = o0 + (size_t)(n - k) * S;
+    if (o0 < a1 && a0 < o1) return fail(c, SS_ERR_INVALID_ARGUMENT, "d_out overlaps d_data");
+    c->h2d = 0;
+    DevGuard g(c->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    try {
+        return dispatch(dt, [&](auto* tag) {
+            typedef std::remove_pointer_t<decltype(tag)> T;
+            return run_upper<T>(c, (const T*)d_data, (u64)n, (u64)k, (T*)d_out, h_result, st);
+        });
+    } catch (...) {
+        return fail(c, SS_ERR_INTERNAL, "exception in ss_select_upper");
+    }
+}
+
+ss_status ss_select_multi(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int32_t m,
+                          const int64_t* h_ks, void* h_results, void* stream) {
+    ss_status rc = check_common(c, dt, d_data, n, 0, h_results);
+    if (rc) return rc;
+    if (!h_ks || m < 1 || m > MULTI_MAX) return fail(c, SS_ERR_INVALID_ARGUMENT, "m must be in [1, 1024], ks non-NULL");
+    for (int i = 0; i < m; ++i)
+        if (h_ks[i] < 0 || h_ks[i] >= n) return fail(c, SS_ERR_INVALID_ARGUMENT, "rank outside [0, n)");
+    if (((uintptr_t)d_data) % dt_size(dt)) return fail(c, SS_ERR_INVALID_ARGUMENT, "d_data misaligned for dtype");
+    c->h2d = 0;
+    DevGuard g(c->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    try {
+        return dispatch(dt, [&](auto* tag) {
+            typedef std::remove_pointer_t<decltype(tag)> T;
+            return run_multi<T>(c, dt, (const T*)d_data, (u64)n, m, h_ks, h_results, st);
+        });
+    } catch (...) {
+        return fail(c, SS_ERR_INTERNAL, "exception in ss_select_multi");
+    }
 }
 
 static ss_status approx_impl(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k, int32_t b,
@@ -1246,6 +1512,20 @@ ss_status ss_step_filter(ss_context* c, ss_dtype dt, const void* d_data, int64_t
         filter_kernel<T><<<grid, K5_THREADS, FILTER_SMEM, st>>>((const T*)d_data, (T*)d_out, f);
         CKLAUNCH("filter_kernel");
         return SS_OK;
+    });
+}
+
+ss_status ss_step_count_ablation(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, const void* d_tree,
+                                 int32_t b, int32_t mode, uint64_t* d_totals, void* stream) {
+    if (!c || !dt_size(dt) || !d_data || !d_tree || !d_totals || n < 1 || !pow2(b) || b < 2 || b > 1024 ||
+        mode < 0 || mode >= ABL_MODES || ((uintptr_t)d_data) % dt_size(dt))
+        return c ? fail(c, SS_ERR_INVALID_ARGUMENT, "ss_step_count_ablation: bad argument") : SS_ERR_INVALID_ARGUMENT;
+    DevGuard g(c->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    CK(cudaMemsetAsync(d_totals, 0, sizeof(u64) * b, st));
+    return dispatch(dt, [&](auto* tag) -> ss_status {
+        typedef std::remove_pointer_t<decltype(tag)> T;
+        return launch_ablation<T>(c, (const T*)d_data, (u64)n, d_tree, log2i(b), mode, (u64*)d_totals, st);
     });
 }
 
