@@ -10,6 +10,9 @@ compares).  This module compiles it with gcc on first use (or ``build()``) and
 marshals numpy arrays through ctypes.  Every function cites the passage of
 ``/root/reference/PAPER.md`` it follows; see the header of ``oracle.c``.
 
+:func:`quickselect` (the NEXT-3 baseline's method mirror) is pure Python on
+top of :func:`select`, :func:`cmp` and :func:`sample_indices`.
+
 Parity status: every function below is pinned in ``tests/test_oracle.py``
 except the approximate *value* of :func:`approx_select`, which has no closed
 form (it depends on the random sample); it is pinned statistically (mean rank
@@ -266,6 +269,55 @@ def sampleselect(data, k: int, b: int, s: int, base_case: int, seed: int, max_le
     if lv < 0:
         raise ValueError("oracle_sampleselect: invalid argument")
     return out[0], levels[:min(lv, max_levels)].tolist()
+
+
+QS_SAMPLE = 1024
+
+
+def quickselect(data, k: int, base_case: int, seed: int, max_levels: int = 128):
+    """QuickSelect, the paper's comparison baseline (§IV.F), in the
+    three-way reading R24 of Fig. 5's branchless bipartition (L375-389):
+    per level, pivot = the median (sorted position 512) of the 1024 keys at
+    the R7 sample indices of the level; one pass over the level puts x < p at
+    out[l++] and x > p at out[r--] and counts x == p; k < L recurses left,
+    L <= k < L + E returns p, else recurses right with k - L - E.  Levels with
+    n <= base_case are finished by sort-and-index (Fig. 1 lines 2-5).
+    Pure Python loop over the elements: small inputs only.  Returns
+    (value, [n_l for every level incl. the last]).  The level order of the
+    GPU's partition is nondeterministic (atomics), so only the result and
+    n_1 (level 0 draws its sample from the caller's array) are comparable."""
+    cur = np.ascontiguousarray(_arr(data))
+    dt = cur.dtype
+    k = int(k)
+    sizes = []
+    for level in range(max_levels):
+        n = cur.size
+        sizes.append(n)
+        if n <= base_case:
+            return select(cur, k), sizes
+        idx = sample_indices(seed, level, n, 0, QS_SAMPLE)
+        p = select(cur[idx], QS_SAMPLE // 2)
+        out = np.empty_like(cur)
+        l, r, eq = 0, n - 1, 0
+        for i in range(n):                   # Fig. 5, three-way (R24)
+            c = cmp(cur[i], p, dt)
+            if c < 0:
+                out[l] = cur[i]
+                l += 1
+            elif c > 0:
+                out[r] = cur[i]
+                r -= 1
+            else:
+                eq += 1
+        L, G = l, n - 1 - r
+        if k < L:
+            cur = out[:L].copy()
+        elif k < L + eq:
+            return _scalar(dt, p)[0], sizes
+        else:
+            cur = out[n - G:].copy()
+            k -= L + eq
+    raise RuntimeError("oracle quickselect: level limit")
 
 
 def sample_size(b: int) -> int:

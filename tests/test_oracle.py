@@ -420,3 +420,51 @@ def test_select_multi_monotone_and_numpy(dtype):
         assert oracle.cmp(a, b, dtype) <= 0
     with pytest.raises(ValueError):
         oracle.select_multi(x, [x.size])
+
+
+# ---- QuickSelect mirror (reading R24) -------
+@settings(max_examples=120, deadline=None)
+@given(st.lists(st.integers(-3, 3), min_size=1, max_size=60), st.data())
+def test_quickselect_mirror_tiny_duplicates(vals, data):
+    """base_case = 0 forces the three-way partition at every level down to a
+    single pivot answer: duplicates exercise the == pivot exit."""
+    x = np.array(vals, dtype=np.int64)
+    k = data.draw(st.integers(0, len(vals) - 1))
+    v, sizes = oracle.quickselect(x, k, base_case=0, seed=3)
+    assert int(v) == sorted(vals)[k] == int(oracle.select_bruteforce(x, k))
+    assert all(a > b for a, b in zip(sizes, sizes[1:]))
+
+
+@settings(max_examples=80, deadline=None)
+@given(st.lists(_f32_special, min_size=1, max_size=30), st.data())
+def test_quickselect_mirror_tiny_special_f32(bits, data):
+    """-0/+0, NaNs, infinities: the partition uses totalOrder (R3)."""
+    x = np.array(bits, dtype=np.uint32).view(np.float32)
+    k = data.draw(st.integers(0, len(bits) - 1))
+    v, _ = oracle.quickselect(x, k, base_case=0, seed=9)
+    assert _bits(v) == _bits(oracle.select_bruteforce(x, k))
+
+
+@pytest.mark.parametrize("kind,dtype", [("uniform", np.float32), ("distinct16", np.float64),
+                                        ("equal", np.int32), ("perm", np.int64)])
+def test_quickselect_mirror_level0_counts(kind, dtype):
+    """Level 0 keeps exactly #{x < p} (left) or #{x > p} (right) elements
+    for the median-of-sample pivot p, and the result is sorted[k]; the
+    median-of-1024 pivot roughly halves continuous data."""
+    n = 3000
+    x = datagen.make(kind, n, dtype, seed=4)
+    idx = oracle.sample_indices(11, 0, n, 0, oracle.QS_SAMPLE)
+    p = oracle.select(x[idx], oracle.QS_SAMPLE // 2)
+    L, Le = oracle.count_less(x, p), oracle.count_leq(x, p)
+    for k in [0, n // 2, n - 1]:
+        v, sizes = oracle.quickselect(x, k, base_case=64, seed=11)
+        assert _bits(v) == _bits(oracle.select(x, k))
+        assert sizes[0] == n
+        if k < L:
+            assert sizes[1] == L
+        elif k >= Le:
+            assert sizes[1] == n - Le
+        else:
+            assert len(sizes) == 1
+    if kind in ("uniform", "perm"):
+        assert abs(L - n / 2) < 0.1 * n
