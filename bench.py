@@ -43,7 +43,7 @@ def parse():
     p.add_argument("--log2n", type=int, default=28, help="elements per GPU = 2^log2n")
     p.add_argument("--dtype", default="float32", choices=["float32", "float64", "int32", "int64"])
     p.add_argument("--kind", default="uniform")
-    p.add_argument("--mode", default="exact", choices=["exact", "approx", "upper", "multi"],
+    p.add_argument("--mode", default="exact", choices=["exact", "approx", "upper", "multi", "quick"],
                    help="upper: top-k fusion (select + all larger elements, §IV.I), k = n - --upper-count")
     p.add_argument("--upper-count", type=int, default=1 << 20, help="upper mode: n - k elements returned")
     p.add_argument("--ranks", type=int, default=8, help="multi mode: number of ranks (seeded, uniform)")
@@ -179,7 +179,7 @@ def run_reference(args, rank, world):
     b = args.b or (256 if kind == "exact" else 1024)
 
     def step():
-        if kind == "exact":
+        if kind in ("exact", "quick"):
             oracle.select(sample, m // 2)
         elif kind == "upper":
             oracle.select_upper(sample, m - min(args.upper_count, m))
@@ -229,7 +229,8 @@ def run_ours(args, rank, world, local_rank):
         ctx.configure(classify=args.classify)
     upper = args.mode == "upper"
     multi = args.mode == "multi"
-    exact = args.mode in ("exact", "upper", "multi")
+    quick = args.mode == "quick"
+    exact = args.mode in ("exact", "upper", "multi", "quick")
     b = args.b or (256 if exact else 1024)
     if exact:
         ctx.configure(b_exact=b)
@@ -247,6 +248,11 @@ def run_ours(args, rank, world, local_rank):
 
         def step(inp):
             return ctx.select_multi(inp, ks)
+    elif quick:
+        k = n // 2
+
+        def step(inp):
+            return ctx.quickselect(inp, k)
     elif upper:
         k = n - args.upper_count
         outbuf = torch.empty(args.upper_count, dtype=xd.dtype, device=xd.device)
@@ -323,7 +329,7 @@ def run_ours(args, rank, world, local_rank):
     # ---- end-to-end through the public API with HOST buffers
     e2e_steps = args.e2e_steps or min(args.steps, 10)
     xhn = xh.numpy()
-    if world == 1 and not upper and not multi:
+    if world == 1 and not upper and not multi and not quick:
         step_h = (lambda: ctx.select(xhn, k)) if exact else (lambda: ctx.approx_select(xhn, k, b))
         step_h()
         torch.cuda.synchronize()
@@ -353,10 +359,11 @@ def run_ours(args, rank, world, local_rank):
     peak, peak_src = measured_peak()
     S = np.dtype(args.dtype).itemsize
     fused0 = exact and bool(last.get("fused_levels", 0) & 1)
-    if multi:
-        kname = "whole call (shared sample + count, bucket extractions, per-rank tails)"
+    if multi or quick:
+        kname = ("whole call (shared sample + count, bucket extractions, per-rank tails)" if multi else
+                 "whole call (QuickSelect baseline: per level pivot + partition + decide, SURVEY NEXT-3)")
         k2_bytes = float(last["bytes_algorithmic"])
-        tkey = f"multi_{args.dtype}_2p{args.log2n}"
+        tkey = f"{args.mode}_{args.dtype}_2p{args.log2n}"
     elif upper:
         kname = "upper_gather_kernel (top-k pass: read the input, write the elements > result)"
         k2_bytes = S * n + S * int(last["upper_greater"])
@@ -369,7 +376,7 @@ def run_ours(args, rank, world, local_rank):
         kname = "count_kernel (K2, level 0)"
         k2_bytes = (S + (1 if exact else 0)) * n          # read S*n, write n oracle bytes
         tkey = f"count_{args.mode}_{args.dtype}_2p{args.log2n}"
-    k2_avg = float(np.mean(upper_ms)) if upper and upper_ms else (ms if multi else kavg(0, 1, prof_timed))
+    k2_avg = float(np.mean(upper_ms)) if upper and upper_ms else (ms if multi or quick else kavg(0, 1, prof_timed))
     achieved = k2_bytes / (k2_avg * 1e-3) / 1e9
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -386,7 +393,8 @@ def run_ours(args, rank, world, local_rank):
         "vs_baseline": None, "dtype": _dt_name(args.dtype), "data": "synthetic",
         "config": {"workload": f"{args.mode} select n=2^{args.log2n} {args.dtype} {args.kind} per GPU, "
                                + (f"k=N-{args.upper_count} (+ all larger elements), b={b}" if upper else
-                                  f"{args.ranks} seeded uniform ranks in one call, b={b}" if multi else f"k=N/2, b={b}"),
+                                  f"{args.ranks} seeded uniform ranks in one call, b={b}" if multi else
+                                  "k=N/2, one median-of-1024 pivot per level" if quick else f"k=N/2, b={b}"),
                    "n_per_gpu": n, "k": k, "b": b, "kind": args.kind,
                    "l2": "inputs larger than L2 (1 GiB input vs 126 MB L2); no flush"},
         "roofline": {"bound": "hbm", "kernel": kname, "achieved": achieved,

@@ -117,7 +117,8 @@ typedef struct {
                                           output is copies of result) */
     float ms_upper_gather;             /* ss_select_upper with profile != 0: device ms of the
                                           upper_gather_kernel pass (CUDA events) */
-    int32_t reserved_stats_;
+    float ms_quick;                    /* ss_quickselect with profile != 0: device ms from the
+                                          init kernel to the last batch (CUDA events) */
 } ss_stats;
 
 /* ---- context --------------------------------------------------------- */
@@ -230,6 +231,24 @@ enum { SS_ABL_SHARED = 0, SS_ABL_SHARED_WA = 1, SS_ABL_SHARED_FIG6 = 2, SS_ABL_G
 ss_status ss_step_count_ablation(ss_context* ctx, ss_dtype dt, const void* d_data, int64_t n,
                                  const void* d_tree, int32_t b, int32_t mode, uint64_t* d_totals,
                                  void* stream);
+
+/* QuickSelect, the paper's own GPU comparison baseline (
+ * §IV.F, Fig. 5, §V.D).  Same result as
+ * ss_select (the element of rank k under totalOrder, 0-based) by a single
+ * pivot per level: the pivot is the median of a 1024-key sample, one pass
+ * splits the level three ways (< pivot to the left of the next buffer,
+ * > pivot to the right, == pivot only counted: reading R24), and the level
+ * recurses into the part holding k or returns the pivot; levels with
+ * n_l <= base_case finish in one CTA.  d_data: caller-owned device array,
+ * read only; n in [1, 2^32).  The context owns two n-element level buffers
+ * (allocated on first use, grown on demand).  Optional outputs:
+ * h_n_level[0..n_level_cap) receives n_l per level (0 past the last one),
+ * *h_levels the number of partition passes.  Synchronises `stream`.
+ * Errors: SS_ERR_INVALID_ARGUMENT for the ss_select conditions, n >= 2^32,
+ * n_level_cap < 0 or a positive cap with NULL h_n_level. */
+ss_status ss_quickselect(ss_context* ctx, ss_dtype dt, const void* d_data, int64_t n, int64_t k,
+                         void* h_result, int64_t* h_n_level, int32_t n_level_cap, int32_t* h_levels,
+                         void* stream);
 
 /* ---- sharded (multi-GPU) selection support -------------------
  * The sharded driver (paper_conf_ipps_ribizela19_b200/sharded.py) runs one

@@ -105,7 +105,7 @@ class Context:
                 "tl_us": [[list(s.tl_us[l][q]) for q in range(3)] for l in range(L + 1)],
                 "spec_levels": s.spec_levels, "fused_levels": s.fused_levels,
                 "lut_ctas": s.lut_ctas, "upper_greater": s.upper_greater,
-                "ms_upper_gather": s.ms_upper_gather}
+                "ms_upper_gather": s.ms_upper_gather, "ms_quick": s.ms_quick}
 
     def raw_tl(self):
         """profile=3: the full 32x3 timeline (us after init; -1 = not stamped)."""
@@ -181,6 +181,23 @@ class Context:
         self._check(self._lib.ss_select_upper(self._h, dt, p, n, int(k), ctypes.c_void_p(out.data_ptr()),
                                               ctypes.c_void_p(val.ctypes.data), self._stream(stream)))
         return val[0], out
+
+    def quickselect(self, x, k: int, stream=None, with_levels: bool = False):
+        """QuickSelect baseline: the same
+        element as select(x, k), by one pivot per level.  x must be a CUDA
+        tensor.  with_levels=True also returns the list of n_l per level."""
+        if not _is_tensor(x):
+            raise TypeError("quickselect takes a CUDA tensor")
+        dt, p, n, npdt, _ = self._args(x)
+        val = np.empty(1, dtype=npdt)
+        cap = 128
+        nl = (ctypes.c_int64 * cap)()
+        lv = ctypes.c_int32(0)
+        self._check(self._lib.ss_quickselect(self._h, dt, p, n, int(k), ctypes.c_void_p(val.ctypes.data),
+                                             nl, cap, ctypes.byref(lv), self._stream(stream)))
+        if with_levels:
+            return val[0], [int(nl[i]) for i in range(lv.value + 1)]
+        return val[0]
 
     def select_multi(self, x, ks, stream=None):
         """Multi-rank selection: the elements of ranks ks

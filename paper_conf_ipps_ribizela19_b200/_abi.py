@@ -23,7 +23,7 @@ EXPORTS = [
     "ss_create", "ss_destroy", "ss_get_config", "ss_set_config", "ss_last_stats", "ss_profile_totals",
     "ss_last_error", "ss_status_string", "ss_abi_version",
     "ss_select", "ss_select_host", "ss_approx_select", "ss_approx_select_host", "ss_select_upper", "ss_select_multi",
-    "ss_step_sample", "ss_step_tree", "ss_step_count", "ss_step_count_ablation", "ss_step_filter",
+    "ss_step_sample", "ss_step_tree", "ss_step_count", "ss_step_count_ablation", "ss_quickselect", "ss_step_filter",
     "ss_step_search", "ss_step_keys_to_values",
 ]
 
@@ -50,7 +50,7 @@ class SSStats(ctypes.Structure):
                 ("lut_ctas", ctypes.c_int32), ("lut_marker", ctypes.c_int32),
                 ("spec_levels", ctypes.c_int32), ("fused_levels", ctypes.c_int32),
                 ("upper_greater", ctypes.c_int64), ("ms_upper_gather", ctypes.c_float),
-                ("reserved_stats_", ctypes.c_int32)]
+                ("ms_quick", ctypes.c_float)]
 
 
 class SSError(RuntimeError):
@@ -95,6 +95,7 @@ def lib() -> ctypes.CDLL:
         L.ss_approx_select.argtypes = [vp, st, vp, i64, i64, i32, vp, ctypes.POINTER(i64), vp]
         L.ss_approx_select_host.argtypes = [vp, st, vp, i64, i64, i32, vp, ctypes.POINTER(i64), vp]
         L.ss_select_upper.argtypes = [vp, st, vp, i64, i64, vp, vp, vp]
+        L.ss_quickselect.argtypes = [vp, st, vp, i64, i64, vp, ctypes.POINTER(i64), i32, ctypes.POINTER(i32), vp]
         L.ss_select_multi.argtypes = [vp, st, vp, i64, i32, ctypes.POINTER(i64), vp, vp]
         L.ss_step_sample.argtypes = [vp, st, vp, i64, i32, i64, i64, vp, vp]
         L.ss_step_tree.argtypes = [vp, st, vp, i32, i32, i32, vp, vp, vp, vp]

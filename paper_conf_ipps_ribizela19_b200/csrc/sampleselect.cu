@@ -23,6 +23,7 @@
 #include <type_traits>
 
 #include "kernels.cuh"
+#include "quickselect.cuh"
 #include "sampleselect.h"
 
 using namespace ss;
@@ -102,6 +103,13 @@ struct ss_context {
     unsigned char* d_multi_scratch = nullptr;
     void* d_multi = nullptr;
     size_t cap_multi = 0;
+    // ss_quickselect: device control block, ping-pong level
+    // buffers (level 0 writes up to n - 1 elements), batch-end host mirror
+    QsCtl* d_qs = nullptr;
+    QsCtl* h_qs = nullptr;
+    void* d_qsbuf[2] = {nullptr, nullptr};
+    size_t cap_qsbuf = 0;
+    cudaEvent_t ev_qs[2] = {nullptr, nullptr};
     bool host_timing = false;
     double ht[5] = {};
     long long ht_n = 0;
@@ -1106,6 +1114,85 @@ ss_status run_multi(ss_context* c, ss_dtype dt, const T* d, u64 n, int m, const 
     return SS_OK;
 }
 
+// QuickSelect baseline (quickselect.cuh).
+// Levels are enqueued in batches of QS_BATCH (pivot -> partition -> decide,
+// each early-exiting once the answer is known); one 8-byte-aligned header
+// copy per batch tells the host whether to enqueue more.
+constexpr int QS_BATCH = 12;
+template <typename T>
+ss_status run_quick(ss_context* c, const T* d, u64 n, u64 k, void* h_result, int64_t* h_n_level, int32_t cap,
+                    int32_t* h_levels, cudaStream_t st) {
+    if (n >= ((u64)1 << 32)) return fail(c, SS_ERR_INVALID_ARGUMENT, "quickselect: n must be < 2^32");
+    if (!c->d_qs) {
+        CK(cudaMalloc(&c->d_qs, sizeof(QsCtl)));
+        CK(cudaMallocHost(&c->h_qs, sizeof(QsCtl)));
+        CK(cudaEventCreate(&c->ev_qs[0]));
+        CK(cudaEventCreate(&c->ev_qs[1]));
+    }
+    const size_t need = (size_t)n * sizeof(T);
+    if (c->cap_qsbuf < need) {
+        for (auto& p : c->d_qsbuf) {
+            cudaFree(p);
+            p = nullptr;
+        }
+        c->cap_qsbuf = 0;
+        CK(cudaMalloc(&c->d_qsbuf[0], need));
+        CK(cudaMalloc(&c->d_qsbuf[1], need));
+        c->cap_qsbuf = need;
+    }
+    const u32 B = (u32)std::min<int64_t>(std::max<int64_t>(c->cfg.base_case, 1), (int64_t)BASE_THREADS * BASE_PT);
+    constexpr int IPT = QP_IPT;
+    const u32 grid = (u32)c->sms * QP_MINB;
+    T* buf[2] = {(T*)c->d_qsbuf[0], (T*)c->d_qsbuf[1]};
+    const bool prof = c->cfg.profile != 0;
+    if (prof) CK(cudaEventRecord(c->ev_qs[0], st));
+    qs_init_kernel<<<1, 1, 0, st>>>(c->d_qs, n, k);
+    CK(cudaGetLastError());
+    int launches = 1, level = 0;
+    for (;;) {
+        for (int q = 0; q < QS_BATCH; ++q, ++level) {
+            const T* bin = buf[(level + 1) & 1];      // level l reads buffer (l-1)&1 (level 0: d)
+            qs_pivot_kernel<T><<<1, 1024, 0, st>>>(d, bin, c->d_qs, B, c->cfg.seed, level);
+            qs_partition_kernel<T, IPT><<<grid, QP_THREADS, 0, st>>>(d, bin, buf[level & 1], c->d_qs, level);
+            qs_decide_kernel<T><<<1, 1, 0, st>>>(c->d_qs, level);
+            CK(cudaGetLastError());
+            launches += 3;
+        }
+        CK(cudaMemcpyAsync(c->h_qs, c->d_qs, offsetof(QsCtl, n_level), cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        if (c->h_qs->done) break;
+        if (level + QS_BATCH > QS_MAX_LEVELS) return fail(c, SS_ERR_INTERNAL, "quickselect: level limit reached");
+    }
+    if (prof) CK(cudaEventRecord(c->ev_qs[1], st));
+    CK(cudaMemcpyAsync(c->h_qs, c->d_qs, sizeof(QsCtl), cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));
+    const QsCtl& h = *c->h_qs;
+    std::memcpy(h_result, &h.bits, sizeof(T));
+    const int lv = (int)h.levels;
+    const int nvalid = lv + (h.eq_exit ? 0 : 1);   // an equality exit has no base-case level
+    double bytes = 0;
+    for (int l = 0; l < lv; ++l) bytes += (double)sizeof(T) * ((double)h.n_level[l] + (double)h.n_out[l]);
+    if (!h.eq_exit) bytes += (double)sizeof(T) * (double)h.n_level[lv];   // base case reads its level
+    if (h_levels) *h_levels = lv;
+    if (h_n_level)
+        for (int l = 0; l < cap && l < QS_MAX_LEVELS; ++l)
+            h_n_level[l] = l < nvalid ? (int64_t)h.n_level[l] : 0;
+    c->stats = ss_stats{};
+    c->stats.levels = std::min(lv, SS_MAX_LEVELS - 1);
+    c->stats.equality_exit = (int)h.eq_exit;
+    for (int l = 0; l < nvalid && l < SS_MAX_LEVELS; ++l) c->stats.n_level[l] = (int64_t)h.n_level[l];
+    c->stats.bytes_algorithmic = bytes;
+    c->stats.launches = launches;
+    c->stats.d2h_bytes = (int64_t)(offsetof(QsCtl, n_level) * (size_t)(level / QS_BATCH) + sizeof(QsCtl));
+    c->launches_total += launches;
+    if (prof) {
+        float ms = 0;
+        CK(cudaEventElapsedTime(&ms, c->ev_qs[0], c->ev_qs[1]));
+        c->stats.ms_quick = ms;
+    }
+    return SS_OK;
+}
+
 ss_status check_common(ss_context* c, ss_dtype dt, const void* p, int64_t n, int64_t k, void* out) {
     if (!c) return SS_ERR_INVALID_ARGUMENT;
     if (!dt_size(dt)) return fail(c, SS_ERR_INVALID_ARGUMENT, "unknown dtype");
@@ -1222,6 +1309,12 @@ void ss_destroy(ss_context* c) {
     cudaFree(c->d_upper_cnt);
     cudaFree(c->d_multi_scratch);
     cudaFree(c->d_multi);
+    cudaFree(c->d_qs);
+    cudaFree(c->d_qsbuf[0]);
+    cudaFree(c->d_qsbuf[1]);
+    if (c->h_qs) cudaFreeHost(c->h_qs);
+    for (auto& e : c->ev_qs)
+        if (e) cudaEventDestroy(e);
     for (auto& e : c->ev_upper)
         if (e) cudaEventDestroy(e);
     for (auto& e : c->graphs) {
@@ -1360,6 +1453,24 @@ ss_status ss_select_upper(ss_context* c, ss_dtype dt, const void* d_data, int64_
         });
     } catch (...) {
         return fail(c, SS_ERR_INTERNAL, "exception in ss_select_upper");
+    }
+}
+
+ss_status ss_quickselect(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k, void* h_result,
+                         int64_t* h_n_level, int32_t n_level_cap, int32_t* h_levels, void* stream) {
+    ss_status rc = check_common(c, dt, d_data, n, k, h_result);
+    if (rc) return rc;
+    if (n_level_cap < 0 || (n_level_cap > 0 && !h_n_level))
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "ss_quickselect: bad n_level buffer");
+    DevGuard g(c->device);
+    try {
+        return dispatch(dt, [&](auto* tag) {
+            typedef std::remove_pointer_t<decltype(tag)> T;
+            return run_quick<T>(c, (const T*)d_data, (u64)n, (u64)k, h_result, h_n_level, n_level_cap, h_levels,
+                                (cudaStream_t)stream);
+        });
+    } catch (...) {
+        return fail(c, SS_ERR_INTERNAL, "exception in ss_quickselect");
     }
 }
 

@@ -1,0 +1,130 @@
+"""GPU parity of the QuickSelect baseline (§IV.F,
+Fig. 5; reading R24: three-way split, pivot = median of a 1024-key
+sample).  ss_quickselect must return exactly the oracle's sorted[k]
+(bit-exact, totalOrder) for every dtype, size and value distribution, and
+its level sizes must strictly shrink (every level drops at least the pivot's
+copies, so the loop terminates)."""
+import numpy as np
+import pytest
+
+import datagen
+import oracle
+
+pytestmark = pytest.mark.gpu
+
+DTYPES = [np.float32, np.float64, np.int32, np.int64]
+
+
+def _bits(v):
+    v = np.asarray(v)
+    u = np.uint32 if v.dtype.itemsize == 4 else np.uint64
+    return int(v.reshape(1).view(u)[0])
+
+
+@pytest.fixture(scope="module")
+def ctx(cuda_device):
+    import paper_conf_ipps_ribizela19_b200 as ss
+    return ss.Context(0)
+
+
+def _dev(x):
+    import torch
+    return torch.from_numpy(np.ascontiguousarray(x)).to("cuda:0")
+
+
+def _gen(kind, n, dtype, seed):
+    if kind in ("uniform", "normal", "exponential", "specials") and np.dtype(dtype).kind == "i":
+        kind = "int"
+    return datagen.make(kind, n, dtype, seed)
+
+
+def _check(ctx, x, xd, k):
+    v, lev = ctx.quickselect(xd, k, with_levels=True)
+    assert _bits(v) == _bits(oracle.select(x, k)), (x.dtype, x.size, k)
+    assert lev[0] == x.size
+    assert all(b < a for a, b in zip(lev, lev[1:]) if b), lev
+    return lev
+
+
+@pytest.mark.parametrize("dtype", DTYPES)
+@pytest.mark.parametrize("n", [1, 2, 3, 17, 1000, 16384, 16385, 65536 + 13, (1 << 20) + 7])
+def test_quick_sizes(ctx, dtype, n):
+    """Base case only, one partition level, several tiles with a ragged tail."""
+    x = _gen("normal", n, dtype, seed=n + 11)
+    xd = _dev(x)
+    for k in sorted({0, n // 2, n - 1, (n * 3) // 7}):
+        _check(ctx, x, xd, k)
+
+
+@pytest.mark.parametrize("dtype", DTYPES)
+@pytest.mark.parametrize("kind", ["uniform", "exponential", "distinct16", "distinct2", "equal", "perm", "specials"])
+def test_quick_kinds(ctx, dtype, kind):
+    """Duplicate-heavy and adversarial inputs: the == pivot part is the early
+    exit (reading R24); specials carry -0/+0, NaNs and infinities (reading R3)."""
+    n = (1 << 18) + 5
+    x = _gen(kind, n, dtype, seed=len(kind) * 31 + 7)
+    xd = _dev(x)
+    for k in [0, 1, n // 3, n // 2, n - 2, n - 1]:
+        _check(ctx, x, xd, k)
+
+
+def test_quick_all_equal_exits_at_level0(ctx):
+    """All-equal input: the sampled pivot is the value, L = G = 0, so level 0
+    answers by the pivot (no base case)."""
+    n = 1 << 20
+    x = np.full(n, 3.25, np.float32)
+    v, lev = ctx.quickselect(_dev(x), n // 2, with_levels=True)
+    assert _bits(v) == _bits(np.float32(3.25))
+    assert ctx.stats()["equality_exit"] is True
+    assert lev[0] == n
+
+
+def test_quick_unaligned_view(ctx):
+    """An input view starting at an odd element offset (no 16-byte alignment)."""
+    import torch
+    x = _gen("uniform", (1 << 19) + 3, np.float32, seed=77)
+    xd = _dev(x)
+    v = ctx.quickselect(xd[1:], 12345)
+    assert _bits(v) == _bits(oracle.select(x[1:], 12345))
+    assert torch.equal(xd.cpu(), torch.from_numpy(x))          # input not modified
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.float64])
+def test_quick_matches_select_large(ctx, dtype):
+    """At 2^24 (a BASELINE config size): same bits as ss_select and as the
+    oracle's count invariant #{x < v} <= k < #{x <= v}."""
+    n = 1 << 24
+    x = _gen("uniform", n, dtype, seed=5)
+    xd = _dev(x)
+    for k in [1, n // 2, n - 1]:
+        v, lev = ctx.quickselect(xd, k, with_levels=True)
+        assert _bits(v) == _bits(ctx.select(xd, k))
+        assert oracle.count_less(x, v) <= k < oracle.count_leq(x, v)
+        assert len(lev) >= 3
+        st = ctx.stats()
+        assert st["bytes_algorithmic"] >= x.itemsize * n
+
+
+def test_quick_bad_args(ctx):
+    import paper_conf_ipps_ribizela19_b200 as ss
+    xd = _dev(np.arange(10, dtype=np.float32))
+    with pytest.raises(ss.SSError):
+        ctx.quickselect(xd, 10)
+    with pytest.raises(ss.SSError):
+        ctx.quickselect(xd, -1)
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.int64])
+def test_quick_level1_size_matches_mirror(ctx, dtype):
+    """Level 0 samples the caller's array with the R7 generator on both sides,
+    so the GPU's n_1 equals the oracle mirror's (later levels see the GPU's
+    atomic-ordered buffers and may pick other pivots)."""
+    n = 20000
+    x = _gen("uniform", n, dtype, seed=8)
+    xd = _dev(x)
+    seed = ctx.config["seed"]
+    for k in [0, n // 2, n - 1]:
+        v, lev = ctx.quickselect(xd, k, with_levels=True)
+        mv, msz = oracle.quickselect(x, k, base_case=16384, seed=seed)
+        assert _bits(v) == _bits(mv)
+        assert lev[:2] == msz[:2], (lev, msz)
