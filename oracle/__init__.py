@@ -271,14 +271,14 @@ def sampleselect(data, k: int, b: int, s: int, base_case: int, seed: int, max_le
     return out[0], levels[:min(lv, max_levels)].tolist()
 
 
-QS_SAMPLE = 1024
+QS_SAMPLE = 256
 
 
 def quickselect(data, k: int, base_case: int, seed: int, max_levels: int = 128):
     """QuickSelect, the paper's comparison baseline (§IV.F), in the
     three-way reading R24 of Fig. 5's branchless bipartition (L375-389):
-    per level, pivot = the median (sorted position 512) of the 1024 keys at
-    the R7 sample indices of the level; one pass over the level puts x < p at
+    per level, pivot = the median (sorted position QS_SAMPLE // 2 = 128) of
+    the QS_SAMPLE = 256 keys at the R7 sample indices of the level; one pass over the level puts x < p at
     out[l++] and x > p at out[r--] and counts x == p; k < L recurses left,
     L <= k < L + E returns p, else recurses right with k - L - E.  Levels with
     n <= base_case are finished by sort-and-index (Fig. 1 lines 2-5).

@@ -450,7 +450,7 @@ def test_quickselect_mirror_tiny_special_f32(bits, data):
 def test_quickselect_mirror_level0_counts(kind, dtype):
     """Level 0 keeps exactly #{x < p} (left) or #{x > p} (right) elements
     for the median-of-sample pivot p, and the result is sorted[k]; the
-    median-of-1024 pivot roughly halves continuous data."""
+    median-of-sample pivot roughly halves continuous data."""
     n = 3000
     x = datagen.make(kind, n, dtype, seed=4)
     idx = oracle.sample_indices(11, 0, n, 0, oracle.QS_SAMPLE)
