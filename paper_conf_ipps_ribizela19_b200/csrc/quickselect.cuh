@@ -14,7 +14,7 @@
 // right, keys == p are only counted (n_l - L - G of them) -- so rank k is
 // either in the left part, equal to the pivot (early exit, like the equality
 // buckets of §IV.C) or in the right part, and every level strictly shrinks.
-// The pivot is the median of a 1024-key sample of the level (the paper does
+// The pivot is the median of a 256-key sample of the level (the paper does
 // not say how it picks the pivot).
 //
 // GPU shape per level l (input n_l, output buffer l & 1):
@@ -33,7 +33,7 @@
 namespace ss {
 
 constexpr int QS_MAX_LEVELS = 128;
-constexpr int QS_SAMPLE = 1024;
+constexpr int QS_SAMPLE = 256;  // pivot = sample median (R24)
 constexpr u32 QP_THREADS = 256;
 constexpr int QP_MINB = 4;      // <= 64 registers: 4 CTAs (1024 threads) per SM
 constexpr int QP_IPT = 16;      // keys per thread: 4096-key tiles
@@ -74,6 +74,7 @@ qs_pivot_kernel(const T* __restrict__ in0, const T* __restrict__ buf_in, QsCtl* 
     __shared__ u32 hist[32 * 256];
     __shared__ u32 misc[16];
     __shared__ K red[64];
+    __shared__ u32 misc_rank[QS_SAMPLE];
     if (c->done) return;
     const u64 n = c->n;
     const T* in = qs_input(in0, buf_in, c, level);
@@ -87,11 +88,31 @@ qs_pivot_kernel(const T* __restrict__ in0, const T* __restrict__ buf_in, QsCtl* 
         }
         return;
     }
+    // the median by stable rank: thread t ranks sample key t & 255 against
+    // the quarter t >> 8 of the sample, the four partial ranks are summed in
+    // shared memory; the key of stable rank QS_SAMPLE / 2 is sorted[QS_SAMPLE / 2]
     const u64 base = level_base(seed, level);    // reading R7
-    block_sort_keys<K>(keys, (u32)QS_SAMPLE, [&](u32 j) { return load_key(in + sample_index(base, j, n)); });
-    if (threadIdx.x == 0) {
+    u32* rank = misc_rank;
+    const u32 t = threadIdx.x & (QS_SAMPLE - 1), part = threadIdx.x / QS_SAMPLE;
+    if (threadIdx.x < QS_SAMPLE) {
+        keys[t] = load_key(in + sample_index(base, t, n));
+        rank[t] = 0;
+    }
+    __syncthreads();
+    if (part < 1024 / QS_SAMPLE) {
+        const K me = keys[t];
+        u32 r = 0;
+        constexpr u32 Q = QS_SAMPLE / (1024 / QS_SAMPLE);
+        for (u32 j = part * Q; j < (part + 1) * Q; ++j) {
+            const K o = keys[j];
+            r += (o < me) | ((o == me) & (j < t));
+        }
+        atomicAdd(&rank[t], r);
+    }
+    __syncthreads();
+    if (threadIdx.x < QS_SAMPLE && rank[t] == QS_SAMPLE / 2) {
         c->n_level[level] = n;
-        c->pivot = (u64)keys[QS_SAMPLE / 2];
+        c->pivot = (u64)keys[t];
         c->lg = 0;
     }
 }

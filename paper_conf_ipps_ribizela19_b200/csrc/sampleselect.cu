@@ -1115,10 +1115,11 @@ ss_status run_multi(ss_context* c, ss_dtype dt, const T* d, u64 n, int m, const 
 }
 
 // QuickSelect baseline (quickselect.cuh).
-// Levels are enqueued in batches of QS_BATCH (pivot -> partition -> decide,
+// Levels are enqueued in batches (the first sized to the expected depth, then
+// QS_BATCH; pivot -> partition -> decide,
 // each early-exiting once the answer is known); one 8-byte-aligned header
 // copy per batch tells the host whether to enqueue more.
-constexpr int QS_BATCH = 12;
+constexpr int QS_BATCH = 4;
 template <typename T>
 ss_status run_quick(ss_context* c, const T* d, u64 n, u64 k, void* h_result, int64_t* h_n_level, int32_t cap,
                     int32_t* h_levels, cudaStream_t st) {
@@ -1148,9 +1149,12 @@ ss_status run_quick(ss_context* c, const T* d, u64 n, u64 k, void* h_result, int
     if (prof) CK(cudaEventRecord(c->ev_qs[0], st));
     qs_init_kernel<<<1, 1, 0, st>>>(c->d_qs, n, k);
     CK(cudaGetLastError());
-    int launches = 1, level = 0;
-    for (;;) {
-        for (int q = 0; q < QS_BATCH; ++q, ++level) {
+    int launches = 1, level = 0, batches = 0;
+    // first batch: the expected depth log2(n / B) + 2 of a median pivot; then QS_BATCH at a time
+    int batch = 2;
+    for (u64 m = n; m > B; m >>= 1) ++batch;
+    for (;; batch = QS_BATCH) {
+        for (int q = 0; q < batch; ++q, ++level) {
             const T* bin = buf[(level + 1) & 1];      // level l reads buffer (l-1)&1 (level 0: d)
             qs_pivot_kernel<T><<<1, 1024, 0, st>>>(d, bin, c->d_qs, B, c->cfg.seed, level);
             qs_partition_kernel<T, IPT><<<grid, QP_THREADS, 0, st>>>(d, bin, buf[level & 1], c->d_qs, level);
@@ -1160,6 +1164,7 @@ ss_status run_quick(ss_context* c, const T* d, u64 n, u64 k, void* h_result, int
         }
         CK(cudaMemcpyAsync(c->h_qs, c->d_qs, offsetof(QsCtl, n_level), cudaMemcpyDeviceToHost, st));
         CK(cudaStreamSynchronize(st));
+        ++batches;
         if (c->h_qs->done) break;
         if (level + QS_BATCH > QS_MAX_LEVELS) return fail(c, SS_ERR_INTERNAL, "quickselect: level limit reached");
     }
@@ -1183,7 +1188,7 @@ ss_status run_quick(ss_context* c, const T* d, u64 n, u64 k, void* h_result, int
     for (int l = 0; l < nvalid && l < SS_MAX_LEVELS; ++l) c->stats.n_level[l] = (int64_t)h.n_level[l];
     c->stats.bytes_algorithmic = bytes;
     c->stats.launches = launches;
-    c->stats.d2h_bytes = (int64_t)(offsetof(QsCtl, n_level) * (size_t)(level / QS_BATCH) + sizeof(QsCtl));
+    c->stats.d2h_bytes = (int64_t)(offsetof(QsCtl, n_level) * (size_t)batches + sizeof(QsCtl));
     c->launches_total += launches;
     if (prof) {
         float ms = 0;

@@ -1,5 +1,5 @@
 """GPU parity of the QuickSelect baseline (§IV.F,
-Fig. 5; reading R24: three-way split, pivot = median of a 1024-key
+Fig. 5; reading R24: three-way split, pivot = median of a 256-key
 sample).  ss_quickselect must return exactly the oracle's sorted[k]
 (bit-exact, totalOrder) for every dtype, size and value distribution, and
 its level sizes must strictly shrink (every level drops at least the pivot's
