@@ -128,3 +128,16 @@ def test_quick_level1_size_matches_mirror(ctx, dtype):
         mv, msz = oracle.quickselect(x, k, base_case=16384, seed=seed)
         assert _bits(v) == _bits(mv)
         assert lev[:2] == msz[:2], (lev, msz)
+
+
+def test_quick_bench_workload_n2p28(ctx):
+    """bench.py --mode quick's configuration (n = 2^28 uniform fp32, k = n/2,
+    same input recipe as the headline bench): the count invariant
+    #{x < v} <= k < #{x <= v} on the oracle, and the same bits as ss_select."""
+    n = 1 << 28
+    x = datagen.uniform(n, np.float32, seed=datagen.dataset_seed(5, 0))
+    xd = _dev(x)
+    for k in [n // 2, datagen.rank(n, 7)]:
+        v = ctx.quickselect(xd, k)
+        assert oracle.count_less(x, v) <= k < oracle.count_leq(x, v), k
+        assert _bits(v) == _bits(ctx.select(xd, k))
