@@ -35,8 +35,17 @@ namespace ss {
 constexpr int QS_MAX_LEVELS = 128;
 constexpr int QS_SAMPLE = 256;  // pivot = sample median (R24)
 constexpr u32 QP_THREADS = 256;
-constexpr int QP_MINB = 4;      // <= 64 registers: 4 CTAs (1024 threads) per SM
-constexpr int QP_IPT = 16;      // keys per thread: 4096-key tiles
+#ifndef SS_QP_MINB
+#define SS_QP_MINB 6
+#endif
+#ifndef SS_QP_IPT
+#define SS_QP_IPT 16
+#endif
+// CTAs per SM: 4-byte keys 6 (<= 40 registers; measured 1.14 vs 1.19 ms at
+// 2^28 with 4), 8-byte keys 4 (<= 64 registers: 6 spills, 2.70 vs 1.78 ms)
+constexpr int QP_MINB = SS_QP_MINB;
+template <typename T> constexpr int qp_minb() { return sizeof(T) == 4 ? QP_MINB : 4; }
+constexpr int QP_IPT = SS_QP_IPT;     // default 16 keys per thread: 4096-key tiles
 
 struct QsCtl {
     u64 n, k, off;               // level input: n_l elements at buffer + off, rank k_l
@@ -127,7 +136,7 @@ qs_pivot_kernel(const T* __restrict__ in0, const T* __restrict__ buf_in, QsCtl* 
 // are copied out with consecutive threads on consecutive addresses.  Order
 // inside a level is unspecified (reading R24).  Padding (i >= n) is neither.
 template <typename T, int IPT>
-__global__ void __launch_bounds__(QP_THREADS, QP_MINB)
+__global__ void __launch_bounds__(QP_THREADS, qp_minb<T>())
 qs_partition_kernel(const T* __restrict__ in0, const T* __restrict__ buf_in, T* __restrict__ out,
                     QsCtl* __restrict__ c, int level) {
     typedef typename Traits<T>::Key K;

@@ -1142,8 +1142,8 @@ ss_status run_quick(ss_context* c, const T* d, u64 n, u64 k, void* h_result, int
         c->cap_qsbuf = need;
     }
     const u32 B = (u32)std::min<int64_t>(std::max<int64_t>(c->cfg.base_case, 1), (int64_t)BASE_THREADS * BASE_PT);
-    constexpr int IPT = QP_IPT;
-    const u32 grid = (u32)c->sms * QP_MINB;
+    constexpr int IPT = (sizeof(T) == 8 && QP_IPT > 16) ? 16 : QP_IPT;   // 8-byte tiles: <= 32 KB static stage
+    const u32 grid = (u32)c->sms * qp_minb<T>();
     T* buf[2] = {(T*)c->d_qsbuf[0], (T*)c->d_qsbuf[1]};
     const bool prof = c->cfg.profile != 0;
     if (prof) CK(cudaEventRecord(c->ev_qs[0], st));
