@@ -394,7 +394,7 @@ def run_ours(args, rank, world, local_rank):
         "config": {"workload": f"{args.mode} select n=2^{args.log2n} {args.dtype} {args.kind} per GPU, "
                                + (f"k=N-{args.upper_count} (+ all larger elements), b={b}" if upper else
                                   f"{args.ranks} seeded uniform ranks in one call, b={b}" if multi else
-                                  "k=N/2, one median-of-1024 pivot per level" if quick else f"k=N/2, b={b}"),
+                                  "k=N/2, one median-of-256-sample pivot per level" if quick else f"k=N/2, b={b}"),
                    "n_per_gpu": n, "k": k, "b": b, "kind": args.kind,
                    "l2": "inputs larger than L2 (1 GiB input vs 126 MB L2); no flush"},
         "roofline": {"bound": "hbm", "kernel": kname, "achieved": achieved,

@@ -57,7 +57,7 @@ typedef struct {
     int32_t b_exact;      /* buckets per exact level: power of two in [4, 256]
                              (oracle bytes cap b at 256, L272-276). default 256 */
     int32_t sample_size;  /* s: 0 = per-b default clamp(16 b, 4096, 16384) (L557-561);
-                             else a power of two in [b, 16384] */
+                             else a power of two in [max(64, b_exact, b_deep), 16384] */
     int32_t base_case;    /* B: levels with n <= B finish in one CTA (L97, L579-583);
                              power of two in [256, 16384]. default 16384 */
     int32_t ctas_per_sm;  /* count/filter grid = ctas_per_sm * #SMs. default 4 */
@@ -200,16 +200,29 @@ ss_status ss_step_sample(ss_context* ctx, ss_dtype dt, const void* d_data, int64
 ss_status ss_step_tree(ss_context* ctx, ss_dtype dt, const void* d_sample_keys, int32_t s, int32_t b,
                        int32_t fixup, void* d_tree, void* d_splitters, uint8_t* d_eq, void* stream);
 
+/* Oracle-byte layout (§IV.B-b: one bucket byte per element).  The
+ * count kernel stores the bytes of 16-byte input vectors as aligned words, so
+ * the byte of element i lives at d_oracles[ss_oracle_offset(dt, d_data, n) + i],
+ * with the offset in [0, 16) chosen so that the bytes of the input's first
+ * 16-byte-aligned element are 16-byte aligned.  An oracle buffer therefore
+ * needs n + 16 bytes and a 16-byte-aligned base.  Pure host arithmetic (no
+ * device access); returns -1 for an unknown dtype. */
+int64_t ss_oracle_offset(ss_dtype dt, const void* d_data, int64_t n);
+
 /* K2 (§IV.B-b, Fig. 4, §IV.G): classify d_data[0..n) against the tree (keys),
  * write per-bucket totals d_totals[b] (uint64, overwritten) and, if
  * d_oracles != NULL (requires b <= 256), the bucket byte of element i to
- * d_oracles[i]. */
+ * d_oracles[ss_oracle_offset(dt, d_data, n) + i] (see above: >= n + 16 bytes,
+ * 16-byte-aligned base, else SS_ERR_INVALID_ARGUMENT).  Also records the
+ * per-CTA counts the next ss_step_filter on the same data needs. */
 ss_status ss_step_count(ss_context* ctx, ss_dtype dt, const void* d_data, int64_t n, const void* d_tree,
                         int32_t b, uint64_t* d_totals, uint8_t* d_oracles, void* stream);
 
-/* K5 (§IV.B-c): stable compaction of the elements i with
- * d_oracles[i] == bucket into d_out (values, input order).  Writes the
- * number of elements copied to *d_count (uint64). */
+/* K5 (§IV.B-c): stable compaction of the elements i with oracle
+ * byte == bucket (layout of ss_oracle_offset; the buffer ss_step_count wrote,
+ * 16-byte-aligned base) into d_out (values, input order).  Must follow
+ * ss_step_count on the same d_data and n (it uses that pass's per-CTA
+ * counts).  Writes the number of elements copied to *d_count (uint64). */
 ss_status ss_step_filter(ss_context* ctx, ss_dtype dt, const void* d_data, int64_t n,
                          const uint8_t* d_oracles, int32_t bucket, void* d_out, uint64_t* d_count,
                          void* stream);

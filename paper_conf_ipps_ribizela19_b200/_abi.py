@@ -24,7 +24,7 @@ EXPORTS = [
     "ss_last_error", "ss_status_string", "ss_abi_version",
     "ss_select", "ss_select_host", "ss_approx_select", "ss_approx_select_host", "ss_select_upper", "ss_select_multi",
     "ss_step_sample", "ss_step_tree", "ss_step_count", "ss_step_count_ablation", "ss_quickselect", "ss_step_filter",
-    "ss_step_search", "ss_step_keys_to_values",
+    "ss_step_search", "ss_step_keys_to_values", "ss_oracle_offset",
 ]
 
 
@@ -104,8 +104,11 @@ def lib() -> ctypes.CDLL:
         L.ss_step_filter.argtypes = [vp, st, vp, i64, vp, i32, vp, vp, vp]
         L.ss_step_search.argtypes = [vp, vp, i32, i64, vp, vp, vp]
         L.ss_step_keys_to_values.argtypes = [vp, st, vp, i64, vp, vp]
+        L.ss_oracle_offset.argtypes = [st, vp, i64]
+        L.ss_oracle_offset.restype = i64
         for name in EXPORTS:
-            if name not in ("ss_destroy", "ss_last_error", "ss_status_string", "ss_abi_version"):
+            if name not in ("ss_destroy", "ss_last_error", "ss_status_string", "ss_abi_version",
+                            "ss_oracle_offset"):
                 getattr(L, name).restype = st
         _lib = L
         return _lib

@@ -3,7 +3,9 @@
     python -m paper_conf_ipps_ribizela19_b200.build [--force] [--verbose]
 
 nvcc cross-compiles without a GPU; the .so is git-ignored but travels to the
-GPU box with the gpurun snapshot.
+GPU box with the gpurun snapshot.  Each translation unit (abi.cu, one
+inst_<dtype>.cu per dtype, sharded.cu) compiles to an object in parallel, then
+nvcc links the shared library.
 """
 from __future__ import annotations
 
@@ -11,18 +13,21 @@ import glob
 import os
 import subprocess
 import sys
+from concurrent.futures import ThreadPoolExecutor
 
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(PKG, "libsampleselect.so")
+OBJ = os.path.join(ROOT, "build", "obj")
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 
 NVCC_FLAGS = [
     "-O3", "-std=c++17", "-gencode", "arch=compute_100a,code=sm_100a", "-lineinfo",
-    "-Xcompiler", "-fPIC", "-shared", "--expt-relaxed-constexpr",
+    "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr", "-diag-suppress", "186",
 ]
+LINK_LIBS = ["-ldl"]
 
 
 def _sources():
@@ -45,14 +50,31 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None) ->
     target = out or LIB
     if not force and out is None and up_to_date():
         return LIB
-    tmp = target + f".tmp{os.getpid()}"
     extra = os.environ.get("SS_NVCC_EXTRA", "").split()
-    cmd = [NVCC, *NVCC_FLAGS, *extra, f"-I{INCLUDE}", "-o", tmp, *_sources()]
-    if verbose:
-        cmd.insert(1, "-Xptxas=-v")
-        print(" ".join(cmd), flush=True)
-    subprocess.check_call(cmd)
-    os.replace(tmp, target)
+    tag = f"{os.getpid()}"
+    os.makedirs(OBJ, exist_ok=True)
+
+    def compile_one(src):
+        obj = os.path.join(OBJ, os.path.basename(src)[:-3] + f".{tag}.o")
+        cmd = [NVCC, *NVCC_FLAGS, *extra, f"-I{INCLUDE}", "-c", "-o", obj, src]
+        if verbose:
+            cmd.insert(1, "-Xptxas=-v")
+            print(" ".join(cmd), flush=True)
+        subprocess.check_call(cmd)
+        return obj
+
+    srcs = _sources()
+    with ThreadPoolExecutor(max_workers=min(len(srcs), os.cpu_count() or 4)) as ex:
+        objs = list(ex.map(compile_one, srcs))
+    tmp = target + f".tmp{tag}"
+    try:
+        subprocess.check_call([NVCC, "-shared", "-gencode", "arch=compute_100a,code=sm_100a", "-o", tmp,
+                               *objs, *LINK_LIBS])
+        os.replace(tmp, target)
+    finally:
+        for o in objs:
+            if os.path.exists(o):
+                os.remove(o)
     return target
 
 

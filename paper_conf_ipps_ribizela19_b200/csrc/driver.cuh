@@ -1,4 +1,11 @@
-// sampleselect.cu -- level driver (Layer 1) and the C ABI (include/sampleselect.h).
+#pragma once
+// driver.cuh -- level driver (Layer 1): the context, the per-call control of
+// the kernels of one SampleSelect level, and the per-dtype operations the C ABI
+// (abi.cu) dispatches to.  Compiled once per dtype (inst_<dtype>.cu defines
+// SS_INST_T before including this file), so the kernel templates of one dtype
+// live in one translation unit and the four build in parallel; abi.cu includes
+// it without SS_INST_T for the context and the shared helpers only.  Everything
+// here has internal linkage except the op_* entry points at the end.
 //
 // The driver follows Fig. 1 (L95-127) with the recursion control kept on the
 // device (§IV.E): per call it enqueues an init kernel and, per
@@ -110,6 +117,8 @@ struct ss_context {
     void* d_qsbuf[2] = {nullptr, nullptr};
     size_t cap_qsbuf = 0;
     cudaEvent_t ev_qs[2] = {nullptr, nullptr};
+    int k2_occ[4][11] = {};          // count_kernel<T, H> resident CTAs per SM (per dtype, H)
+    bool kw_attr[4][2] = {};         // window_kernel<T, APX> shared-memory attribute set
     bool host_timing = false;
     double ht[5] = {};
     long long ht_n = 0;
@@ -119,9 +128,6 @@ static inline double now_us() {
 }
 
 static constexpr u32 MAX_GRID = 2048;
-// SS_CARVEOUT (build flag): force one shared-memory carveout on every kernel
-// of the chain.  Off by default: measured slower -- an all-shared carveout
-// leaves L1 too small for the count kernel's in-flight 128-bit loads.
 static constexpr int MAX_S = 16384;
 // sample sizes up to this are ranked by the wide K1 (s/32 CTAs, s^2 pairs);
 // larger samples (approximate b = 1024) use the one-CTA bitonic K1
@@ -219,23 +225,21 @@ ss_status grow(ss_context* c, void** p, size_t* cap, size_t need) {
 }
 
 // count/filter grid: resident CTAs of the count kernel x #SMs (one wave)
+// (the occupancy is cached per context: a context belongs to one device and
+// one host thread, so no cache is shared between threads)
 template <typename T, int H>
 u32 count_grid(ss_context* c) {
-    static int occ[64] = {0};
-    int dev = c->device & 63;
-    if (!occ[dev]) {
+    int& occ = c->k2_occ[dt_code<T>() - 1][H];
+    if (!occ) {
         int o = 0;
         typedef typename Traits<T>::Key K;
         cudaFuncSetAttribute(count_kernel<T, H>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                              (int)count_smem_bytes<H, K>());
-#ifdef SS_CARVEOUT
-        cudaFuncSetAttribute(count_kernel<T, H>, cudaFuncAttributePreferredSharedMemoryCarveout, SS_CARVEOUT);
-#endif
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, count_kernel<T, H>, K2_THREADS,
                                                       count_smem_bytes<H, K>());
-        occ[dev] = o > 0 ? o : 1;
+        occ = o > 0 ? o : 1;
     }
-    u32 per = (u32)std::max(1, std::min(c->cfg.ctas_per_sm, occ[dev]));
+    u32 per = (u32)std::max(1, std::min(c->cfg.ctas_per_sm, occ));
     return std::min<u32>(per * (u32)c->sms, MAX_GRID);
 }
 
@@ -261,11 +265,11 @@ ss_status launch_count(ss_context* c, int H, const T* in, CountArgs& a, cudaStre
 template <typename T, bool APX = false>
 ss_status launch_window(ss_context* c, int /*H*/, const T* in, CountArgs a, cudaStream_t st) {
     a.grid = (u32)c->sms * (u32)KW_MINB;
-    static bool attr_set[64] = {};
-    if (!attr_set[c->device & 63]) {
+    bool& attr_set = c->kw_attr[dt_code<T>() - 1][APX ? 1 : 0];
+    if (!attr_set) {
         CK(cudaFuncSetAttribute(window_kernel<T, APX>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)KW_STASH));
-        attr_set[c->device & 63] = true;
+        attr_set = true;
     }
     CK(launch_pdl(window_kernel<T, APX>, dim3(a.grid), dim3(KW_THREADS), KW_STASH, st, in, a));
     CKLAUNCH("window_kernel");
@@ -299,8 +303,6 @@ ss_status set_k1_attrs(ss_context* c) {
     typedef typename Traits<T>::Key K;
     CK(cudaFuncSetAttribute(sample_tree_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                             (int)(16384 * sizeof(K))));
-    CK(cudaFuncSetAttribute(tree_from_keys_kernel<K>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                            (int)(16384 * sizeof(K))));
     CK(cudaFuncSetAttribute(filter_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)FILTER_SMEM));
     CK(cudaFuncSetAttribute(sample_rank_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                             (int)(16384 * sizeof(K))));
@@ -308,14 +310,6 @@ ss_status set_k1_attrs(ss_context* c) {
                             (int)(K1C_CHUNK * sizeof(K))));
     CK(cudaFuncSetAttribute(sample_merge_rank_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                             (int)(16384 * sizeof(K))));
-    // one carveout (all shared) for every kernel of the path: no L1/shared
-    // reconfiguration between consecutive kernels
-#ifdef SS_CARVEOUT
-    CK(cudaFuncSetAttribute(sample_tree_kernel<T>, cudaFuncAttributePreferredSharedMemoryCarveout, SS_CARVEOUT));
-    CK(cudaFuncSetAttribute(filter_kernel<T>, cudaFuncAttributePreferredSharedMemoryCarveout, SS_CARVEOUT));
-    CK(cudaFuncSetAttribute(sample_rank_kernel<T>, cudaFuncAttributePreferredSharedMemoryCarveout, SS_CARVEOUT));
-    CK(cudaFuncSetAttribute(init_kernel<T>, cudaFuncAttributePreferredSharedMemoryCarveout, SS_CARVEOUT));
-#endif
     return SS_OK;
 }
 
@@ -479,7 +473,7 @@ ss_status launch_k1_wide(ss_context* c, const T* in, int lev, int s, u32 B, cuda
     typedef typename Traits<T>::Key K;
     K* sorted = reinterpret_cast<K*>(c->d_sorted) + (size_t)lev * MAX_S;
     mark(c, lev, 0, 0, st);
-    CK(launch_pdl(sample_rank_kernel<T>, dim3((u32)s / 32u), dim3(K1R_THREADS),
+    CK(launch_pdl(sample_rank_kernel<T>, dim3(((u32)s + 31u) / 32u), dim3(K1R_THREADS),
                   k1_smem<T>(s, B), st,
                   in, c->d_ctl + lev, c->d_res, sorted, s, B, (u64)c->cfg.seed, lev,
                   reinterpret_cast<const K*>(presampled)));
@@ -545,7 +539,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     // totals of every planned level are zeroed by init; levels beyond the plan
     // (the rare "incomplete" fallback) are zeroed before they run
     auto enqueue_init = [&](cudaStream_t q) -> ss_status {
-        CK(launch_pdl(init_kernel<T>, dim3(pre0 ? (u32)s / 256u : 1u), dim3(256), 0, q, c->d_ctl,
+        CK(launch_pdl(init_kernel<T>, dim3(pre0 ? ((u32)s + 255u) / 256u : 1u), dim3(256), 0, q, c->d_ctl,
                       (int)(SS_MAX_LEVELS + 1), c->d_totals, (int)((L + 1) * MAX_B), c->d_res, n, k, tl_on, d, s,
                       (u64)c->cfg.seed, sample0));
         CKLAUNCH("init_kernel");
@@ -822,7 +816,7 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     const bool merge = s > WIDE_K1_MAX_S && s % (int)K1C_CHUNK == 0;   // chunk sort + merge rank
     const bool wide = s <= WIDE_K1_MAX_S || merge;
     K* sample0 = s <= WIDE_K1_MAX_S ? reinterpret_cast<K*>(c->d_sample0) : nullptr;
-    CK(launch_pdl(init_kernel<T>, dim3(sample0 ? (u32)s / 256u : 1u), dim3(256), 0, st, c->d_ctl, 2, c->d_totals,
+    CK(launch_pdl(init_kernel<T>, dim3(sample0 ? ((u32)s + 255u) / 256u : 1u), dim3(256), 0, st, c->d_ctl, 2, c->d_totals,
                   (int)MAX_B, c->d_res, n, k, (int)(c->cfg.profile == 3), d, s, (u64)c->cfg.seed, sample0));
     CKLAUNCH("init_kernel");
     ++c->launches;
@@ -984,8 +978,8 @@ ss_status run_upper(ss_context* c, const T* d, u64 n, u64 k, T* d_out, void* h_r
 constexpr int MULTI_MAX = 1024;
 constexpr u64 MULTI_MIN_N = (u64)1 << 20;   // below: one select per rank is cheaper
 // Below 4 ranks the per-rank fused selects win: measured at n = 2^28 fp32
-// (profiles/r01f_next_rows.md) the shared path costs ~0.50 ms + ~0.18 ms per
-// extra rank, a fused single select 0.28 ms.
+// (profiles/r01f_bench_multi1.json, profiles/r01f_bench_multi8.json) the shared
+// path costs ~0.50 ms + ~0.18 ms per extra rank, a fused single select 0.28 ms.
 constexpr int MULTI_MIN_M = 4;
 
 template <typename T>
@@ -1198,479 +1192,8 @@ ss_status run_quick(ss_context* c, const T* d, u64 n, u64 k, void* h_result, int
     return SS_OK;
 }
 
-ss_status check_common(ss_context* c, ss_dtype dt, const void* p, int64_t n, int64_t k, void* out) {
-    if (!c) return SS_ERR_INVALID_ARGUMENT;
-    if (!dt_size(dt)) return fail(c, SS_ERR_INVALID_ARGUMENT, "unknown dtype");
-    if (!p || !out) return fail(c, SS_ERR_INVALID_ARGUMENT, "NULL pointer");
-    if (n < 1) return fail(c, SS_ERR_INVALID_ARGUMENT, "n must be >= 1");
-    if (k < 0 || k >= n) return fail(c, SS_ERR_INVALID_ARGUMENT, "k must be in [0, n)");
-    if (((uintptr_t)p) % dt_size(dt)) return fail(c, SS_ERR_INVALID_ARGUMENT, "data not naturally aligned");
-    return SS_OK;
-}
 
-template <typename F>
-ss_status dispatch(ss_dtype dt, F&& f) {
-    switch (dt) {
-    case SS_FLOAT32: return f((float*)nullptr);
-    case SS_FLOAT64: return f((double*)nullptr);
-    case SS_INT32: return f((int*)nullptr);
-    case SS_INT64: return f((long long*)nullptr);
-    default: return SS_ERR_INVALID_ARGUMENT;
-    }
-}
-
-ss_status stage_host(ss_context* c, const void* h, size_t bytes, cudaStream_t st) {
-    ss_status rc = grow(c, &c->d_stage, &c->cap_stage, bytes);
-    if (rc) return rc;
-    CK(cudaMemcpyAsync(c->d_stage, h, bytes, cudaMemcpyHostToDevice, st));
-    c->h2d = (int64_t)bytes;
-    return SS_OK;
-}
 
 }  // namespace
 
-// =========================================================== C ABI ========
-extern "C" {
-
-int ss_abi_version(void) { return SS_ABI_VERSION; }
-
-const char* ss_status_string(ss_status s) {
-    switch (s) {
-    case SS_OK: return "SS_OK";
-    case SS_ERR_INVALID_ARGUMENT: return "SS_ERR_INVALID_ARGUMENT";
-    case SS_ERR_CUDA: return "SS_ERR_CUDA";
-    case SS_ERR_OUT_OF_MEMORY: return "SS_ERR_OUT_OF_MEMORY";
-    case SS_ERR_INTERNAL: return "SS_ERR_INTERNAL";
-    default: return "SS_UNKNOWN_STATUS";
-    }
-}
-
-ss_status ss_create(int device, ss_context** out) {
-    if (!out || device < 0) return SS_ERR_INVALID_ARGUMENT;
-    *out = nullptr;
-    int ndev = 0;
-    if (cudaGetDeviceCount(&ndev) != cudaSuccess || device >= ndev) {
-        (void)cudaGetLastError();
-        return SS_ERR_CUDA;
-    }
-    ss_context* c = new (std::nothrow) ss_context();
-    if (!c) return SS_ERR_OUT_OF_MEMORY;
-    c->device = device;
-    c->host_timing = std::getenv("SS_HOST_TIMING") != nullptr;
-    c->cfg.b_exact = 256;
-    c->cfg.b_deep = 0;
-    c->cfg.sample_size = 0;
-    c->cfg.base_case = 16384;
-    c->cfg.ctas_per_sm = 4;
-    c->cfg.profile = 0;
-    c->cfg.seed = 0x5A17;
-    c->cfg.classify = 0;
-    c->cfg.fused_filter = 1;
-    c->cfg.spec_z = 3.0f;
-    c->cfg.spec_min_n = (int64_t)1 << 22;
-    c->cfg.spec_max_frac = 0.25f;
-    DevGuard g(device);
-    if (cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess) {
-        (void)cudaGetLastError();
-        delete c;
-        return SS_ERR_CUDA;
-    }
-    ss_status rc = ensure_small(c);
-    if (!rc) rc = set_k1_attrs<float>(c);
-    if (!rc) rc = set_k1_attrs<double>(c);
-    if (!rc) rc = set_k1_attrs<int>(c);
-    if (!rc) rc = set_k1_attrs<long long>(c);
-    if (rc) {
-        ss_destroy(c);
-        return rc;
-    }
-    *out = c;
-    return SS_OK;
-}
-
-void ss_destroy(ss_context* c) {
-    if (!c) return;
-    if (c->host_timing && c->ht_n)
-        std::fprintf(stderr, "ss host timing (us/call over %lld exact calls): prep %.2f graph-launch %.2f "
-                     "wait %.2f post %.2f total %.2f\n", c->ht_n, c->ht[0] / c->ht_n, c->ht[1] / c->ht_n,
-                     c->ht[2] / c->ht_n, c->ht[3] / c->ht_n, c->ht[4] / c->ht_n);
-    DevGuard g(c->device);
-    cudaFree(c->d_oracles);
-    cudaFree(c->d_buf[0]);
-    cudaFree(c->d_buf[1]);
-    cudaFree(c->d_stage);
-    cudaFree(c->d_ctl);
-    cudaFree(c->d_res);
-    cudaFree(c->d_totals);
-    cudaFree(c->d_cta_counts);
-    cudaFree(c->d_tree);
-    cudaFree(c->d_spl);
-    cudaFree(c->d_eq);
-    cudaFree(c->d_sorted);
-    cudaFree(c->d_sample0);
-    cudaFree(c->d_presample);
-    cudaFree(c->d_image);
-    cudaFree(c->d_seq);
-    cudaFree(c->d_upper_cnt);
-    cudaFree(c->d_multi_scratch);
-    cudaFree(c->d_multi);
-    cudaFree(c->d_qs);
-    cudaFree(c->d_qsbuf[0]);
-    cudaFree(c->d_qsbuf[1]);
-    if (c->h_qs) cudaFreeHost(c->h_qs);
-    for (auto& e : c->ev_qs)
-        if (e) cudaEventDestroy(e);
-    for (auto& e : c->ev_upper)
-        if (e) cudaEventDestroy(e);
-    for (auto& e : c->graphs) {
-        if (e.exec) cudaGraphExecDestroy(e.exec);
-        if (e.graph) cudaGraphDestroy(e.graph);
-    }
-    if (c->cap_st) cudaStreamDestroy(c->cap_st);
-    if (c->h_res) cudaFreeHost(c->h_res);
-    if (c->ev_ready)
-        for (int l = 0; l < SS_MAX_LEVELS; ++l)
-            for (int q = 0; q < 3; ++q)
-                for (int e = 0; e < 2; ++e) cudaEventDestroy(c->ev[l][q][e]);
-    (void)cudaGetLastError();
-    delete c;
-}
-
-ss_status ss_get_config(const ss_context* c, ss_config* out) {
-    if (!c || !out) return SS_ERR_INVALID_ARGUMENT;
-    *out = c->cfg;
-    return SS_OK;
-}
-
-ss_status ss_set_config(ss_context* c, const ss_config* cfg) {
-    if (!c || !cfg) return SS_ERR_INVALID_ARGUMENT;
-    if (!pow2(cfg->b_exact) || cfg->b_exact < 4 || cfg->b_exact > 256)
-        return fail(c, SS_ERR_INVALID_ARGUMENT, "b_exact must be a power of two in [4, 256]");
-    if (cfg->b_deep != 0 && (!pow2(cfg->b_deep) || cfg->b_deep < 4 || cfg->b_deep > 256))
-        return fail(c, SS_ERR_INVALID_ARGUMENT, "b_deep must be 0 or a power of two in [4, 256]");
-    if (cfg->sample_size != 0 && (!pow2(cfg->sample_size) || cfg->sample_size > 16384 ||
-                                  cfg->sample_size < std::max(cfg->b_exact, cfg->b_deep)))
-        return fail(c, SS_ERR_INVALID_ARGUMENT, "sample_size must be 0 or a power of two in [b, 16384]");
-    if (!pow2(cfg->base_case) || cfg->base_case < 256 || cfg->base_case > 16384)
-        return fail(c, SS_ERR_INVALID_ARGUMENT, "base_case must be a power of two in [256, 16384]");
-    if (cfg->profile < 0 || cfg->profile > 3)
-        return fail(c, SS_ERR_INVALID_ARGUMENT, "profile must be 0, 1, 2 or 3");
-    if (cfg->classify < 0 || cfg->classify > 1)
-        return fail(c, SS_ERR_INVALID_ARGUMENT, "classify must be 0 (auto) or 1 (tree walk)");
-    if (cfg->ctas_per_sm < 1 || cfg->ctas_per_sm > 16)
-        return fail(c, SS_ERR_INVALID_ARGUMENT, "ctas_per_sm must be in [1, 16]");
-    if (cfg->fused_filter < 0 || cfg->fused_filter > 1)
-        return fail(c, SS_ERR_INVALID_ARGUMENT, "fused_filter must be 0 or 1");
-    if (!(cfg->spec_z >= 0.0f && cfg->spec_z <= 64.0f))
-        return fail(c, SS_ERR_INVALID_ARGUMENT, "spec_z must be in [0, 64]");
-    if (cfg->spec_min_n < 1)
-        return fail(c, SS_ERR_INVALID_ARGUMENT, "spec_min_n must be >= 1");
-    if (!(cfg->spec_max_frac > 0.0f && cfg->spec_max_frac <= 1.0f))
-        return fail(c, SS_ERR_INVALID_ARGUMENT, "spec_max_frac must be in (0, 1]");
-    // captured graphs bake in grid sizes and the fused-filter parameters
-    const bool regrid = cfg->ctas_per_sm != c->cfg.ctas_per_sm || cfg->classify != c->cfg.classify ||
-                        cfg->fused_filter != c->cfg.fused_filter || cfg->spec_z != c->cfg.spec_z ||
-                        cfg->spec_min_n != c->cfg.spec_min_n || cfg->spec_max_frac != c->cfg.spec_max_frac;
-    c->cfg = *cfg;
-    if (regrid)                   // captured grid sizes are stale (the other knobs are part of the graph key)
-        for (auto& e : c->graphs) {
-            if (e.exec) cudaGraphExecDestroy(e.exec);
-            if (e.graph) cudaGraphDestroy(e.graph);
-            e = ss_context::GraphEntry();
-        }
-    return SS_OK;
-}
-
-ss_status ss_profile_totals(ss_context* c, double* ms_sum, int64_t* count, int64_t* launches,
-                            int64_t* calls, int32_t reset) {
-    if (!c) return SS_ERR_INVALID_ARGUMENT;
-    for (int l = 0; l < SS_MAX_LEVELS; ++l)
-        for (int q = 0; q < 3; ++q) {
-            if (ms_sum) ms_sum[l * 3 + q] = c->prof_sum[l][q];
-            if (count) count[l * 3 + q] = c->prof_cnt[l][q];
-            if (reset) { c->prof_sum[l][q] = 0; c->prof_cnt[l][q] = 0; }
-        }
-    if (launches) *launches = c->launches_total;
-    if (calls) *calls = c->calls_total;
-    if (reset) { c->launches_total = 0; c->calls_total = 0; }
-    return SS_OK;
-}
-
-ss_status ss_last_stats(const ss_context* c, ss_stats* out) {
-    if (!c || !out) return SS_ERR_INVALID_ARGUMENT;
-    *out = c->stats;
-    return SS_OK;
-}
-
-const char* ss_last_error(const ss_context* c) { return c ? c->err.c_str() : "NULL context"; }
-
-static ss_status select_impl(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k,
-                             void* h_result, void* stream);
-
-ss_status ss_select(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k, void* h_result,
-                    void* stream) {
-    if (c) c->h2d = 0;
-    return select_impl(c, dt, d_data, n, k, h_result, stream);
-}
-
-static ss_status select_impl(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k,
-                             void* h_result, void* stream) {
-    ss_status rc = check_common(c, dt, d_data, n, k, h_result);
-    if (rc) return rc;
-    DevGuard g(c->device);
-    cudaStream_t st = (cudaStream_t)stream;
-    try {
-        return dispatch(dt, [&](auto* tag) {
-            typedef std::remove_pointer_t<decltype(tag)> T;
-            return run_exact<T>(c, (const T*)d_data, (u64)n, (u64)k, h_result, st);
-        });
-    } catch (...) {
-        return fail(c, SS_ERR_INTERNAL, "exception in ss_select");
-    }
-}
-
-ss_status ss_select_host(ss_context* c, ss_dtype dt, const void* h_data, int64_t n, int64_t k,
-                         void* h_result, void* stream) {
-    ss_status rc = check_common(c, dt, h_data, n, k, h_result);
-    if (rc) return rc;
-    DevGuard g(c->device);
-    cudaStream_t st = (cudaStream_t)stream;
-    if ((rc = stage_host(c, h_data, (size_t)n * dt_size(dt), st))) return rc;
-    return select_impl(c, dt, c->d_stage, n, k, h_result, stream);
-}
-
-ss_status ss_select_upper(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k, void* d_out,
-                          void* h_result, void* stream) {
-    ss_status rc = check_common(c, dt, d_data, n, k, h_result);
-    if (rc) return rc;
-    if (!d_out) return fail(c, SS_ERR_INVALID_ARGUMENT, "d_out is NULL");
-    const size_t S = dt_size(dt);
-    const uintptr_t a0 = (uintptr_t)d_data, a1 = a0 + (size_t)n * S, o0 = (uintptr_t)d_out,
-                    o1 = o0 + (size_t)(n - k) * S;
-    if (o0 < a1 && a0 < o1) return fail(c, SS_ERR_INVALID_ARGUMENT, "d_out overlaps d_data");
-    c->h2d = 0;
-    DevGuard g(c->device);
-    cudaStream_t st = (cudaStream_t)stream;
-    try {
-        return dispatch(dt, [&](auto* tag) {
-            typedef std::remove_pointer_t<decltype(tag)> T;
-            return run_upper<T>(c, (const T*)d_data, (u64)n, (u64)k, (T*)d_out, h_result, st);
-        });
-    } catch (...) {
-        return fail(c, SS_ERR_INTERNAL, "exception in ss_select_upper");
-    }
-}
-
-ss_status ss_quickselect(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k, void* h_result,
-                         int64_t* h_n_level, int32_t n_level_cap, int32_t* h_levels, void* stream) {
-    ss_status rc = check_common(c, dt, d_data, n, k, h_result);
-    if (rc) return rc;
-    if (n_level_cap < 0 || (n_level_cap > 0 && !h_n_level))
-        return fail(c, SS_ERR_INVALID_ARGUMENT, "ss_quickselect: bad n_level buffer");
-    DevGuard g(c->device);
-    try {
-        return dispatch(dt, [&](auto* tag) {
-            typedef std::remove_pointer_t<decltype(tag)> T;
-            return run_quick<T>(c, (const T*)d_data, (u64)n, (u64)k, h_result, h_n_level, n_level_cap, h_levels,
-                                (cudaStream_t)stream);
-        });
-    } catch (...) {
-        return fail(c, SS_ERR_INTERNAL, "exception in ss_quickselect");
-    }
-}
-
-ss_status ss_select_multi(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int32_t m,
-                          const int64_t* h_ks, void* h_results, void* stream) {
-    ss_status rc = check_common(c, dt, d_data, n, 0, h_results);
-    if (rc) return rc;
-    if (!h_ks || m < 1 || m > MULTI_MAX) return fail(c, SS_ERR_INVALID_ARGUMENT, "m must be in [1, 1024], ks non-NULL");
-    for (int i = 0; i < m; ++i)
-        if (h_ks[i] < 0 || h_ks[i] >= n) return fail(c, SS_ERR_INVALID_ARGUMENT, "rank outside [0, n)");
-    if (((uintptr_t)d_data) % dt_size(dt)) return fail(c, SS_ERR_INVALID_ARGUMENT, "d_data misaligned for dtype");
-    c->h2d = 0;
-    DevGuard g(c->device);
-    cudaStream_t st = (cudaStream_t)stream;
-    try {
-        return dispatch(dt, [&](auto* tag) {
-            typedef std::remove_pointer_t<decltype(tag)> T;
-            return run_multi<T>(c, dt, (const T*)d_data, (u64)n, m, h_ks, h_results, st);
-        });
-    } catch (...) {
-        return fail(c, SS_ERR_INTERNAL, "exception in ss_select_multi");
-    }
-}
-
-static ss_status approx_impl(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k, int32_t b,
-                             void* h_result, int64_t* h_rank, void* stream);
-
-ss_status ss_approx_select(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k, int32_t b,
-                           void* h_result, int64_t* h_rank, void* stream) {
-    if (c) c->h2d = 0;
-    return approx_impl(c, dt, d_data, n, k, b, h_result, h_rank, stream);
-}
-
-static ss_status approx_impl(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int64_t k, int32_t b,
-                             void* h_result, int64_t* h_rank, void* stream) {
-    ss_status rc = check_common(c, dt, d_data, n, k, h_result);
-    if (rc) return rc;
-    if (!pow2(b) || b < 4 || b > 1024) return fail(c, SS_ERR_INVALID_ARGUMENT, "b must be a power of two in [4, 1024]");
-    DevGuard g(c->device);
-    cudaStream_t st = (cudaStream_t)stream;
-    try {
-        return dispatch(dt, [&](auto* tag) {
-            typedef std::remove_pointer_t<decltype(tag)> T;
-            return run_approx<T>(c, (const T*)d_data, (u64)n, (u64)k, b, h_result, h_rank, st);
-        });
-    } catch (...) {
-        return fail(c, SS_ERR_INTERNAL, "exception in ss_approx_select");
-    }
-}
-
-ss_status ss_approx_select_host(ss_context* c, ss_dtype dt, const void* h_data, int64_t n, int64_t k,
-                                int32_t b, void* h_result, int64_t* h_rank, void* stream) {
-    ss_status rc = check_common(c, dt, h_data, n, k, h_result);
-    if (rc) return rc;
-    DevGuard g(c->device);
-    cudaStream_t st = (cudaStream_t)stream;
-    if ((rc = stage_host(c, h_data, (size_t)n * dt_size(dt), st))) return rc;
-    return approx_impl(c, dt, c->d_stage, n, k, b, h_result, h_rank, stream);
-}
-
-// ------------------------------------------------------------- steps ------
-ss_status ss_step_sample(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, int32_t level,
-                         int64_t slot_begin, int64_t count, void* d_sample_keys, void* stream) {
-    if (!c || !dt_size(dt) || !d_data || !d_sample_keys || n < 1 || count < 0 || slot_begin < 0 || level < 0)
-        return c ? fail(c, SS_ERR_INVALID_ARGUMENT, "ss_step_sample: bad argument") : SS_ERR_INVALID_ARGUMENT;
-    if (count == 0) return SS_OK;
-    DevGuard g(c->device);
-    cudaStream_t st = (cudaStream_t)stream;
-    return dispatch(dt, [&](auto* tag) -> ss_status {
-        typedef std::remove_pointer_t<decltype(tag)> T;
-        typedef typename Traits<T>::Key K;
-        u32 blocks = (u32)std::min<int64_t>((count + 255) / 256, 1024);
-        sample_keys_kernel<T><<<blocks, 256, 0, st>>>((const T*)d_data, (u64)n, level, (u64)slot_begin,
-                                                      (u64)count, c->cfg.seed, (K*)d_sample_keys);
-        CKLAUNCH("sample_keys_kernel");
-        return SS_OK;
-    });
-}
-
-ss_status ss_step_tree(ss_context* c, ss_dtype dt, const void* d_sample_keys, int32_t s, int32_t b,
-                       int32_t fixup, void* d_tree, void* d_splitters, uint8_t* d_eq, void* stream) {
-    if (!c || !dt_size(dt) || !d_sample_keys || !d_tree || !pow2(s) || s > 16384 || !pow2(b) || b < 2 ||
-        b > 1024 || s < b)
-        return c ? fail(c, SS_ERR_INVALID_ARGUMENT, "ss_step_tree: bad argument") : SS_ERR_INVALID_ARGUMENT;
-    DevGuard g(c->device);
-    cudaStream_t st = (cudaStream_t)stream;
-    if (dt_size(dt) == 4) {
-        tree_from_keys_kernel<u32><<<1, K1_THREADS, (size_t)s * 4, st>>>(
-            (const u32*)d_sample_keys, s, b, fixup, (u32*)d_tree, (u32*)d_splitters, d_eq);
-    } else {
-        tree_from_keys_kernel<u64><<<1, K1_THREADS, (size_t)s * 8, st>>>(
-            (const u64*)d_sample_keys, s, b, fixup, (u64*)d_tree, (u64*)d_splitters, d_eq);
-    }
-    CKLAUNCH("tree_from_keys_kernel");
-    return SS_OK;
-}
-
-ss_status ss_step_count(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, const void* d_tree,
-                        int32_t b, uint64_t* d_totals, uint8_t* d_oracles, void* stream) {
-    if (!c || !dt_size(dt) || !d_data || !d_tree || !d_totals || n < 1 || !pow2(b) || b < 4 || b > 1024 ||
-        (d_oracles && b > 256) || ((uintptr_t)d_data) % dt_size(dt))
-        return c ? fail(c, SS_ERR_INVALID_ARGUMENT, "ss_step_count: bad argument") : SS_ERR_INVALID_ARGUMENT;
-    DevGuard g(c->device);
-    cudaStream_t st = (cudaStream_t)stream;
-    ss_status rc = ensure_small(c);
-    if (rc) return rc;
-    CK(cudaMemsetAsync(d_totals, 0, sizeof(u64) * b, st));
-    return dispatch(dt, [&](auto* tag) -> ss_status {
-        typedef std::remove_pointer_t<decltype(tag)> T;
-        CountArgs a{};
-        a.tree = d_tree;
-        a.oracles = d_oracles;
-        a.cta_counts = c->d_cta_counts;
-        a.totals = (u64*)d_totals;
-        a.lut = c->cfg.classify == 0;
-        a.n = (u64)n;
-        a.tail = TAIL_NONE;
-        ss_status r2 = launch_count<T>(c, log2i(b), (const T*)d_data, a, st);
-        if (r2) return r2;
-        c->step_ptr = d_data;
-        c->step_n = (u64)n;
-        c->step_b = b;
-        c->step_dt = (int)dt;
-        c->step_grid = a.grid;
-        return SS_OK;
-    });
-}
-
-ss_status ss_step_filter(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, const uint8_t* d_oracles,
-                         int32_t bucket, void* d_out, uint64_t* d_count, void* stream) {
-    if (!c || !dt_size(dt) || !d_data || !d_oracles || !d_out || !d_count || n < 1 || bucket < 0)
-        return c ? fail(c, SS_ERR_INVALID_ARGUMENT, "ss_step_filter: bad argument") : SS_ERR_INVALID_ARGUMENT;
-    if (c->step_ptr != d_data || c->step_n != (u64)n || c->step_dt != (int)dt || bucket >= c->step_b)
-        return fail(c, SS_ERR_INVALID_ARGUMENT,
-                    "ss_step_filter must follow ss_step_count on the same data (per-CTA counts)");
-    DevGuard g(c->device);
-    cudaStream_t st = (cudaStream_t)stream;
-    const u32 grid = c->step_grid;
-    return dispatch(dt, [&](auto* tag) -> ss_status {
-        typedef std::remove_pointer_t<decltype(tag)> T;
-        CK(cudaMemsetAsync(d_count, 0, sizeof(u64), st));
-        FilterArgs f{};
-        f.oracles = d_oracles;
-        f.cta_counts = c->d_cta_counts;
-        f.b_count = (u32)c->step_b;
-        f.count_out = (u64*)d_count;
-        f.n = (u64)n;
-        f.bucket = (u32)bucket;
-        f.grid = grid;
-        filter_kernel<T><<<grid, K5_THREADS, FILTER_SMEM, st>>>((const T*)d_data, (T*)d_out, f);
-        CKLAUNCH("filter_kernel");
-        return SS_OK;
-    });
-}
-
-ss_status ss_step_count_ablation(ss_context* c, ss_dtype dt, const void* d_data, int64_t n, const void* d_tree,
-                                 int32_t b, int32_t mode, uint64_t* d_totals, void* stream) {
-    if (!c || !dt_size(dt) || !d_data || !d_tree || !d_totals || n < 1 || !pow2(b) || b < 2 || b > 1024 ||
-        mode < 0 || mode >= ABL_MODES || ((uintptr_t)d_data) % dt_size(dt))
-        return c ? fail(c, SS_ERR_INVALID_ARGUMENT, "ss_step_count_ablation: bad argument") : SS_ERR_INVALID_ARGUMENT;
-    DevGuard g(c->device);
-    cudaStream_t st = (cudaStream_t)stream;
-    CK(cudaMemsetAsync(d_totals, 0, sizeof(u64) * b, st));
-    return dispatch(dt, [&](auto* tag) -> ss_status {
-        typedef std::remove_pointer_t<decltype(tag)> T;
-        return launch_ablation<T>(c, (const T*)d_data, (u64)n, d_tree, log2i(b), mode, (u64*)d_totals, st);
-    });
-}
-
-ss_status ss_step_search(ss_context* c, const uint64_t* d_totals, int32_t b, int64_t k, const uint8_t* d_eq,
-                         int64_t* d_out, void* stream) {
-    if (!c || !d_totals || !d_out || b < 1 || b > 1024 || k < 0)
-        return c ? fail(c, SS_ERR_INVALID_ARGUMENT, "ss_step_search: bad argument") : SS_ERR_INVALID_ARGUMENT;
-    DevGuard g(c->device);
-    cudaStream_t st = (cudaStream_t)stream;
-    search_kernel<<<1, 256, 0, st>>>((const u64*)d_totals, (u32)b, (u64)k, d_eq, (long long*)d_out);
-    CKLAUNCH("search_kernel");
-    return SS_OK;
-}
-
-ss_status ss_step_keys_to_values(ss_context* c, ss_dtype dt, const void* d_keys, int64_t count, void* d_values,
-                                 void* stream) {
-    if (!c || !dt_size(dt) || !d_keys || !d_values || count < 0)
-        return c ? fail(c, SS_ERR_INVALID_ARGUMENT, "ss_step_keys_to_values: bad argument") : SS_ERR_INVALID_ARGUMENT;
-    if (count == 0) return SS_OK;
-    DevGuard g(c->device);
-    cudaStream_t st = (cudaStream_t)stream;
-    u32 blocks = (u32)std::min<int64_t>((count + 255) / 256, 4096);
-    return dispatch(dt, [&](auto* tag) -> ss_status {
-        typedef std::remove_pointer_t<decltype(tag)> T;
-        typedef typename Traits<T>::Key K;
-        keys_to_values_kernel<T><<<blocks, 256, 0, st>>>((const K*)d_keys, (u64)count, (K*)d_values);
-        CKLAUNCH("keys_to_values_kernel");
-        return SS_OK;
-    });
-}
-
-}  // extern "C"
+#include "ops.cuh"

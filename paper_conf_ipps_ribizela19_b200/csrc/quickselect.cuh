@@ -57,7 +57,7 @@ struct QsCtl {
     u64 n_out[QS_MAX_LEVELS];    // L + G written by level l's partition
 };
 
-__global__ void qs_init_kernel(QsCtl* c, u64 n, u64 k) {
+static __global__ void qs_init_kernel(QsCtl* c, u64 n, u64 k) {
     c->n = n;
     c->k = k;
     c->off = 0;
