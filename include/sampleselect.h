@@ -37,7 +37,7 @@
 extern "C" {
 #endif
 
-#define SS_ABI_VERSION 4
+#define SS_ABI_VERSION 5
 #define SS_MAX_LEVELS 32
 
 typedef enum { SS_FLOAT32 = 0, SS_FLOAT64 = 1, SS_INT32 = 2, SS_INT64 = 3 } ss_dtype;
@@ -47,10 +47,12 @@ typedef enum {
     SS_ERR_INVALID_ARGUMENT = 1, /* NULL pointer, n < 1, k not in [0,n), bad dtype/b/config */
     SS_ERR_CUDA = 2,             /* a CUDA runtime error (no device, launch failure, ...) */
     SS_ERR_OUT_OF_MEMORY = 3,    /* workspace allocation failed */
+    SS_ERR_NCCL = 4,             /* NCCL unavailable or a NCCL call failed (sharded calls) */
     SS_ERR_INTERNAL = 5          /* recursion-depth guard tripped (should not happen) */
 } ss_status;
 
 typedef struct ss_context ss_context;
+typedef struct ss_local_group ss_local_group;   /* in-process rank group (sharded calls, tests) */
 
 /* Tuning knobs (§IV.H).  ss_create fills the defaults. */
 typedef struct {
@@ -85,7 +87,9 @@ typedef struct {
     int64_t spec_min_n;   /* levels with at least this many elements speculate. default 2^22 */
     float spec_max_frac;  /* speculate only if the window holds at most this fraction of the
                              sample. default 0.25 */
-    int32_t reserved_;
+    int32_t shard_gather_log2; /* ss_select_sharded: survivors are gathered onto every rank once
+                             the level holds at most 2^shard_gather_log2 elements (then the
+                             single-GPU levels finish); 0 = default 20, else in [12, 28] */
 } ss_config;
 
 /* Per-call statistics of the last ss_select / ss_approx_select. */
@@ -119,6 +123,13 @@ typedef struct {
                                           upper_gather_kernel pass (CUDA events) */
     float ms_quick;                    /* ss_quickselect with profile != 0: device ms from the
                                           init kernel to the last batch (CUDA events) */
+    int32_t incomplete_rounds;         /* ss_select: times the planned levels ended with more than
+                                          base_case elements left and the host enqueued one more
+                                          level (an unlucky sample; 0 almost always) */
+    int32_t shard_levels;              /* ss_select_sharded: sharded levels run before the gather
+                                          (n_level[l] for l < shard_levels are global sizes,
+                                          n_level[shard_levels] the gathered size) */
+    int32_t shard_ranks;               /* ss_select_sharded: ranks of the communicator */
 } ss_stats;
 
 /* ---- context --------------------------------------------------------- */
@@ -278,6 +289,58 @@ ss_status ss_step_search(ss_context* ctx, const uint64_t* d_totals, int32_t b, i
 /* Inverse key map: turn `count` keys into values of dtype dt (in place OK). */
 ss_status ss_step_keys_to_values(ss_context* ctx, ss_dtype dt, const void* d_keys, int64_t count,
                                  void* d_values, void* stream);
+
+/* ---- sharded (multi-GPU) exact selection --------------------
+ * One process (or, with a local group, one host thread) per rank, one context
+ * per rank.  Every rank holds a contiguous shard d_shard[0..n_local) (device,
+ * naturally aligned, read only; n_local >= 0, shards may be empty or of
+ * different sizes) and calls ss_select_sharded with the SAME k_global; every
+ * rank receives the element of rank k_global (0-based, reading R3) of the
+ * union of all shards in *h_result.  Per level every rank draws its share of
+ * the level's sample (proportional to its share of the level), the sample keys
+ * are exchanged so every rank sorts the identical sample and derives the
+ * identical window (reading R21), each rank streams its own shard through the
+ * fused count+filter kernel, and the per-rank counts {below, window} -- the
+ * level's bucket counts -- are exchanged so every rank takes the identical
+ * decision on the device.  Once the level holds at most
+ * 2^shard_gather_log2 elements the survivors are gathered onto every rank and
+ * the single-GPU levels finish.  Exchanges are sum-allreduces over buffers in
+ * which each rank fills disjoint slots.  No host round trip until the result.
+ * Synchronises `stream`.  Errors: SS_ERR_INVALID_ARGUMENT (no communicator,
+ * NULL pointers, k_global outside [0, sum of n_local)), SS_ERR_NCCL, as
+ * ss_select otherwise.  Every rank must make the same sequence of sharded
+ * calls (the exchanges are collective). */
+
+/* NCCL unique id (128 bytes) for ss_comm_init; rank 0 creates it and the
+ * caller broadcasts it (e.g. torch.distributed).  NCCL is loaded at run time
+ * (libnccl.so.2, or $SS_NCCL_LIB); SS_ERR_NCCL if unavailable. */
+ss_status ss_nccl_unique_id(char out_id[128]);
+
+/* Bind a NCCL communicator of `nranks` ranks to the context (collective over
+ * all ranks, each on its context's device).  Replaces a previous one. */
+ss_status ss_comm_init(ss_context* ctx, const char id[128], int nranks, int rank);
+
+/* In-process group of `nranks` (<= 16) ranks: contexts in different host
+ * threads of one process (same device, or peer-accessible devices) exchange
+ * through device-to-device reads with host barriers.  For tests of the
+ * sharded path on one GPU ("virtual ranks"); not graph-capturable. */
+ss_status ss_local_group_create(int nranks, ss_local_group** out);
+void      ss_local_group_destroy(ss_local_group* group);
+ss_status ss_comm_init_local(ss_context* ctx, ss_local_group* group, int rank);
+
+ss_status ss_select_sharded(ss_context* ctx, ss_dtype dt, const void* d_shard, int64_t n_local,
+                            int64_t k_global, void* h_result, void* stream);
+
+/* ---- convenience calls mirroring north_star's select(data, n, k) ---------
+ * A thread-local default context per current CUDA device (created on first
+ * use), the current device's legacy default stream, device input, host
+ * result.  Same semantics and errors as ss_select / ss_approx_select. */
+ss_status ss_select_f32(const float* d_data, int64_t n, int64_t k, float* h_result);
+ss_status ss_select_f64(const double* d_data, int64_t n, int64_t k, double* h_result);
+ss_status ss_select_i32(const int32_t* d_data, int64_t n, int64_t k, int32_t* h_result);
+ss_status ss_select_i64(const int64_t* d_data, int64_t n, int64_t k, int64_t* h_result);
+ss_status ss_approx_select_f32(const float* d_data, int64_t n, int64_t k, int32_t b, float* h_result,
+                               int64_t* h_rank);
 
 #ifdef __cplusplus
 }

@@ -24,7 +24,7 @@ import numpy as np
 from . import _abi
 from ._abi import SSConfig, SSError, SSStats
 
-__all__ = ["Context", "select", "approx_select", "default_context", "SSError"]
+__all__ = ["Context", "LocalGroup", "select", "approx_select", "default_context", "nccl_unique_id", "SSError"]
 
 _NP_DT = {np.dtype(np.float32): _abi.SS_FLOAT32, np.dtype(np.float64): _abi.SS_FLOAT64,
           np.dtype(np.int32): _abi.SS_INT32, np.dtype(np.int64): _abi.SS_INT64}
@@ -105,7 +105,9 @@ class Context:
                 "tl_us": [[list(s.tl_us[l][q]) for q in range(3)] for l in range(L + 1)],
                 "spec_levels": s.spec_levels, "fused_levels": s.fused_levels,
                 "lut_ctas": s.lut_ctas, "upper_greater": s.upper_greater,
-                "ms_upper_gather": s.ms_upper_gather, "ms_quick": s.ms_quick}
+                "ms_upper_gather": s.ms_upper_gather, "ms_quick": s.ms_quick,
+                "incomplete_rounds": s.incomplete_rounds, "shard_levels": s.shard_levels,
+                "shard_ranks": s.shard_ranks}
 
     def raw_tl(self):
         """profile=3: the full 32x3 timeline (us after init; -1 = not stamped)."""
@@ -212,6 +214,36 @@ class Context:
                                               ctypes.c_void_p(out.ctypes.data), self._stream(stream)))
         return out
 
+    # ------------------------------------------------ sharded (§8e) -------
+    def comm_init(self, unique_id: bytes, nranks: int, rank: int):
+        """Bind a NCCL communicator (collective over all ranks; unique_id from
+        nccl_unique_id() on one rank, broadcast by the caller)."""
+        if len(unique_id) != 128:
+            raise ValueError("unique_id must be 128 bytes")
+        self._check(self._lib.ss_comm_init(self._h, ctypes.c_char_p(bytes(unique_id)), int(nranks), int(rank)))
+
+    def comm_init_local(self, group: "LocalGroup", rank: int):
+        """Bind rank `rank` of an in-process group (virtual ranks, one host
+        thread per rank)."""
+        self._check(self._lib.ss_comm_init_local(self._h, group._h, int(rank)))
+
+    def select_sharded(self, x, k: int, stream=None):
+        """Element of rank k (0-based) of the union of every rank's shard x
+        (a 1-D CUDA tensor, may be empty); collective: every rank calls it
+        with the same k and gets the same result."""
+        if not _is_tensor(x):
+            raise TypeError("select_sharded takes a CUDA tensor")
+        if x.numel() == 0:
+            if not x.is_cuda or x.dim() != 1:
+                raise ValueError("input must be a 1-D CUDA tensor")
+            dt, p, n, npdt = _torch_dt(x), ctypes.c_void_p(0), 0, _NP_OF[_torch_dt(x)]
+        else:
+            dt, p, n, npdt, _ = self._args(x)
+        out = np.empty(1, dtype=npdt)
+        self._check(self._lib.ss_select_sharded(self._h, dt, p, n, int(k), ctypes.c_void_p(out.ctypes.data),
+                                                self._stream(stream)))
+        return out[0]
+
     # -------------------------------------------- single steps (tensors) --
     def step_sample(self, x, level: int, slot_begin: int, count: int, out_keys, stream=None):
         dt, p, n, _, _ = self._args(x)
@@ -252,10 +284,50 @@ class Context:
                                              ctypes.c_void_p(eq.data_ptr() if eq is not None else 0),
                                              ctypes.c_void_p(out.data_ptr()), self._stream(stream)))
 
+    def oracle_offset(self, x) -> int:
+        """Offset of element 0's oracle byte in an oracle buffer for x
+        (ss_oracle_offset: byte i lives at offset + i)."""
+        dt, p, n, _, _ = self._args(x)
+        return int(self._lib.ss_oracle_offset(dt, p, n))
+
     def step_keys_to_values(self, dt_code: int, keys, values, stream=None):
         self._check(self._lib.ss_step_keys_to_values(self._h, dt_code, ctypes.c_void_p(keys.data_ptr()),
                                                      keys.numel(), ctypes.c_void_p(values.data_ptr()),
                                                      self._stream(stream)))
+
+
+class LocalGroup:
+    """An in-process rank group (ss_local_group): contexts in different host
+    threads exchange through device memory -- virtual ranks on one GPU."""
+
+    def __init__(self, nranks: int):
+        self._lib = _abi.lib()
+        self._h = ctypes.c_void_p()
+        rc = self._lib.ss_local_group_create(int(nranks), ctypes.byref(self._h))
+        if rc:
+            raise SSError(rc, f"ss_local_group_create({nranks})")
+        self.nranks = int(nranks)
+
+    def close(self):
+        if self._h:
+            self._lib.ss_local_group_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):  # pragma: no cover
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def nccl_unique_id() -> bytes:
+    """A NCCL unique id (128 bytes) for Context.comm_init."""
+    buf = ctypes.create_string_buffer(128)
+    lib = _abi.lib()
+    rc = lib.ss_nccl_unique_id(buf)
+    if rc:
+        raise SSError(rc, "ss_nccl_unique_id: NCCL unavailable")
+    return buf.raw
 
 
 _tls = threading.local()

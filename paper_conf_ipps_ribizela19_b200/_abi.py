@@ -16,7 +16,7 @@ SS_FLOAT32, SS_FLOAT64, SS_INT32, SS_INT64 = 0, 1, 2, 3
 SS_MAX_LEVELS = 32
 ABLATION_MODES = {"shared": 0, "shared_wa": 1, "shared_fig6": 2, "global": 3, "global_wa": 4}
 STATUS = {0: "SS_OK", 1: "SS_ERR_INVALID_ARGUMENT", 2: "SS_ERR_CUDA",
-          3: "SS_ERR_OUT_OF_MEMORY", 5: "SS_ERR_INTERNAL"}
+          3: "SS_ERR_OUT_OF_MEMORY", 4: "SS_ERR_NCCL", 5: "SS_ERR_INTERNAL"}
 
 # every symbol include/sampleselect.h declares
 EXPORTS = [
@@ -25,6 +25,8 @@ EXPORTS = [
     "ss_select", "ss_select_host", "ss_approx_select", "ss_approx_select_host", "ss_select_upper", "ss_select_multi",
     "ss_step_sample", "ss_step_tree", "ss_step_count", "ss_step_count_ablation", "ss_quickselect", "ss_step_filter",
     "ss_step_search", "ss_step_keys_to_values", "ss_oracle_offset",
+    "ss_nccl_unique_id", "ss_comm_init", "ss_local_group_create", "ss_local_group_destroy", "ss_comm_init_local",
+    "ss_select_sharded", "ss_select_f32", "ss_select_f64", "ss_select_i32", "ss_select_i64", "ss_approx_select_f32",
 ]
 
 
@@ -35,7 +37,7 @@ class SSConfig(ctypes.Structure):
                 ("classify", ctypes.c_int32), ("seed", ctypes.c_uint64),
                 ("fused_filter", ctypes.c_int32), ("spec_z", ctypes.c_float),
                 ("spec_min_n", ctypes.c_int64), ("spec_max_frac", ctypes.c_float),
-                ("reserved_", ctypes.c_int32)]
+                ("shard_gather_log2", ctypes.c_int32)]
 
 
 class SSStats(ctypes.Structure):
@@ -50,7 +52,8 @@ class SSStats(ctypes.Structure):
                 ("lut_ctas", ctypes.c_int32), ("lut_marker", ctypes.c_int32),
                 ("spec_levels", ctypes.c_int32), ("fused_levels", ctypes.c_int32),
                 ("upper_greater", ctypes.c_int64), ("ms_upper_gather", ctypes.c_float),
-                ("ms_quick", ctypes.c_float)]
+                ("ms_quick", ctypes.c_float), ("incomplete_rounds", ctypes.c_int32),
+                ("shard_levels", ctypes.c_int32), ("shard_ranks", ctypes.c_int32)]
 
 
 class SSError(RuntimeError):
@@ -105,10 +108,20 @@ def lib() -> ctypes.CDLL:
         L.ss_step_search.argtypes = [vp, vp, i32, i64, vp, vp, vp]
         L.ss_step_keys_to_values.argtypes = [vp, st, vp, i64, vp, vp]
         L.ss_oracle_offset.argtypes = [st, vp, i64]
+        L.ss_nccl_unique_id.argtypes = [ctypes.c_char_p]
+        L.ss_comm_init.argtypes = [vp, ctypes.c_char_p, ctypes.c_int, ctypes.c_int]
+        L.ss_local_group_create.argtypes = [ctypes.c_int, pctx]
+        L.ss_local_group_destroy.argtypes = [vp]
+        L.ss_local_group_destroy.restype = None
+        L.ss_comm_init_local.argtypes = [vp, vp, ctypes.c_int]
+        L.ss_select_sharded.argtypes = [vp, st, vp, i64, i64, vp, vp]
+        for name in ("ss_select_f32", "ss_select_f64", "ss_select_i32", "ss_select_i64"):
+            getattr(L, name).argtypes = [vp, i64, i64, vp]
+        L.ss_approx_select_f32.argtypes = [vp, i64, i64, i32, vp, ctypes.POINTER(i64)]
         L.ss_oracle_offset.restype = i64
         for name in EXPORTS:
             if name not in ("ss_destroy", "ss_last_error", "ss_status_string", "ss_abi_version",
-                            "ss_oracle_offset"):
+                            "ss_oracle_offset", "ss_local_group_destroy"):
                 getattr(L, name).restype = st
         _lib = L
         return _lib

@@ -48,6 +48,7 @@ const char* ss_status_string(ss_status s) {
     case SS_ERR_INVALID_ARGUMENT: return "SS_ERR_INVALID_ARGUMENT";
     case SS_ERR_CUDA: return "SS_ERR_CUDA";
     case SS_ERR_OUT_OF_MEMORY: return "SS_ERR_OUT_OF_MEMORY";
+    case SS_ERR_NCCL: return "SS_ERR_NCCL";
     case SS_ERR_INTERNAL: return "SS_ERR_INTERNAL";
     default: return "SS_UNKNOWN_STATUS";
     }
@@ -77,6 +78,7 @@ ss_status ss_create(int device, ss_context** out) {
     c->cfg.spec_z = 3.0f;
     c->cfg.spec_min_n = (int64_t)1 << 22;
     c->cfg.spec_max_frac = 0.25f;
+    c->cfg.shard_gather_log2 = 0;
     DevGuard g(device);
     if (cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess) {
         (void)cudaGetLastError();
@@ -107,6 +109,10 @@ void ss_destroy(ss_context* c) {
                      "wait %.2f post %.2f total %.2f\n", c->ht_n, c->ht[0] / c->ht_n, c->ht[1] / c->ht_n,
                      c->ht[2] / c->ht_n, c->ht[3] / c->ht_n, c->ht[4] / c->ht_n);
     DevGuard g(c->device);
+    delete c->comm;
+    cudaFree(c->d_dist);
+    cudaFree(c->d_gather[0]);
+    cudaFree(c->d_gather[1]);
     cudaFree(c->d_oracles);
     cudaFree(c->d_buf[0]);
     cudaFree(c->d_buf[1]);
@@ -179,6 +185,8 @@ ss_status ss_set_config(ss_context* c, const ss_config* cfg) {
         return fail(c, SS_ERR_INVALID_ARGUMENT, "spec_min_n must be >= 1");
     if (!(cfg->spec_max_frac > 0.0f && cfg->spec_max_frac <= 1.0f))
         return fail(c, SS_ERR_INVALID_ARGUMENT, "spec_max_frac must be in (0, 1]");
+    if (cfg->shard_gather_log2 != 0 && (cfg->shard_gather_log2 < 12 || cfg->shard_gather_log2 > 28))
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "shard_gather_log2 must be 0 or in [12, 28]");
     // captured graphs bake in grid sizes and the fused-filter parameters
     const bool regrid = cfg->ctas_per_sm != c->cfg.ctas_per_sm || cfg->classify != c->cfg.classify ||
                         cfg->fused_filter != c->cfg.fused_filter || cfg->spec_z != c->cfg.spec_z ||
@@ -467,6 +475,114 @@ ss_status ss_step_keys_to_values(ss_context* c, ss_dtype dt, const void* d_keys,
         typedef std::remove_pointer_t<decltype(tag)> T;
         return op_keys_to_values(c, (const T*)nullptr, d_keys, (u64)count, d_values, st);
     });
+}
+
+// ------------------------------------------------------------ sharded ----
+ss_status ss_nccl_unique_id(char out_id[128]) {
+    if (!out_id) return SS_ERR_INVALID_ARGUMENT;
+    std::string err;
+    return ss_comm::nccl_unique_id(out_id, err);
+}
+
+ss_status ss_comm_init(ss_context* c, const char id[128], int nranks, int rank) {
+    if (!c) return SS_ERR_INVALID_ARGUMENT;
+    if (!id || nranks < 1 || nranks > DIST_MAX_RANKS || rank < 0 || rank >= nranks)
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "ss_comm_init: bad id, nranks (1..16) or rank");
+    ss_status rc = SS_OK;
+    std::string err;
+    ss_comm::ShardComm* comm = ss_comm::make_nccl_comm(id, nranks, rank, c->device, &rc, err);
+    if (!comm) return fail(c, rc, err);
+    delete c->comm;
+    c->comm = comm;
+    return SS_OK;
+}
+
+ss_status ss_local_group_create(int nranks, ss_local_group** out) { return ss_comm::local_group_create(nranks, out); }
+
+void ss_local_group_destroy(ss_local_group* g) { ss_comm::local_group_destroy(g); }
+
+ss_status ss_comm_init_local(ss_context* c, ss_local_group* g, int rank) {
+    if (!c) return SS_ERR_INVALID_ARGUMENT;
+    ss_status rc = SS_OK;
+    std::string err;
+    ss_comm::ShardComm* comm = ss_comm::make_local_comm(g, rank, c->device, &rc, err);
+    if (!comm) return fail(c, rc, err);
+    delete c->comm;
+    c->comm = comm;
+    return SS_OK;
+}
+
+ss_status ss_select_sharded(ss_context* c, ss_dtype dt, const void* d_shard, int64_t n_local, int64_t k_global,
+                            void* h_result, void* stream) {
+    if (!c) return SS_ERR_INVALID_ARGUMENT;
+    if (!dt_size(dt)) return fail(c, SS_ERR_INVALID_ARGUMENT, "unknown dtype");
+    if (!h_result || (n_local > 0 && !d_shard)) return fail(c, SS_ERR_INVALID_ARGUMENT, "NULL pointer");
+    if (n_local < 0 || k_global < 0) return fail(c, SS_ERR_INVALID_ARGUMENT, "n_local and k_global must be >= 0");
+    if (((uintptr_t)d_shard) % dt_size(dt)) return fail(c, SS_ERR_INVALID_ARGUMENT, "data not naturally aligned");
+    if (!c->comm) return fail(c, SS_ERR_INVALID_ARGUMENT, "ss_select_sharded: no communicator (ss_comm_init first)");
+    c->h2d = 0;
+    DevGuard g(c->device);
+    cudaStream_t st = (cudaStream_t)stream;
+    try {
+        return dispatch(dt, [&](auto* tag) {
+            typedef std::remove_pointer_t<decltype(tag)> T;
+            return op_sharded(c, (const T*)d_shard, (u64)n_local, (u64)k_global, h_result, st);
+        });
+    } catch (...) {
+        return fail(c, SS_ERR_INTERNAL, "exception in ss_select_sharded");
+    }
+}
+
+// --------------------------------------------------------- convenience ----
+}  // extern "C"
+
+namespace {
+// thread-local default contexts, one per device (destroyed with the thread)
+struct DefaultContexts {
+    ss_context* ctx[64] = {};
+    ~DefaultContexts() {
+        for (auto* c : ctx)
+            if (c) ss_destroy(c);
+    }
+};
+ss_status default_context(ss_context** out) {
+    thread_local DefaultContexts dc;
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess) {
+        (void)cudaGetLastError();
+        return SS_ERR_CUDA;
+    }
+    if (dev < 0 || dev >= 64) return SS_ERR_INVALID_ARGUMENT;
+    if (!dc.ctx[dev]) {
+        const ss_status rc = ss_create(dev, &dc.ctx[dev]);
+        if (rc) return rc;
+    }
+    *out = dc.ctx[dev];
+    return SS_OK;
+}
+}  // namespace
+
+extern "C" {
+
+#define SS_CONVENIENCE(name, T, DT)                                                       \
+    ss_status name(const T* d_data, int64_t n, int64_t k, T* h_result) {                  \
+        ss_context* c = nullptr;                                                          \
+        const ss_status rc = default_context(&c);                                         \
+        if (rc) return rc;                                                                \
+        return ss_select(c, DT, d_data, n, k, h_result, nullptr);                         \
+    }
+SS_CONVENIENCE(ss_select_f32, float, SS_FLOAT32)
+SS_CONVENIENCE(ss_select_f64, double, SS_FLOAT64)
+SS_CONVENIENCE(ss_select_i32, int32_t, SS_INT32)
+SS_CONVENIENCE(ss_select_i64, int64_t, SS_INT64)
+#undef SS_CONVENIENCE
+
+ss_status ss_approx_select_f32(const float* d_data, int64_t n, int64_t k, int32_t b, float* h_result,
+                               int64_t* h_rank) {
+    ss_context* c = nullptr;
+    const ss_status rc = default_context(&c);
+    if (rc) return rc;
+    return ss_approx_select(c, SS_FLOAT32, d_data, n, k, b, h_result, h_rank, nullptr);
 }
 
 }  // extern "C"

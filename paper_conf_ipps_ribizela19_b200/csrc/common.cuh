@@ -81,6 +81,13 @@ struct LevelCtl {
     u32 spec_eq;    // the window is one equality bucket (§IV.C): a hit returns its value
     u32 pre;        // this level's sample keys were gathered ahead (init / previous level's tail)
     u32 pad2_;
+    // sharded driver (sharded.cuh): n above is this rank's share
+    // of the level, gn the level's size over all ranks (0 = one GPU)
+    u64 gn;
+    u32 pass;       // the level is a pass-through (the global level is already small)
+    u32 directed;   // the window is [klo, klo + kspan) from the previous level's miss, not the sample
+    float dfrac;    // directed window: expected fraction of the level inside it
+    u32 pad3_;
 };
 
 struct SelectResult {
@@ -97,7 +104,7 @@ struct SelectResult {
     unsigned int fused_levels;// bit l: level l's survivors came from the fused filter (window hit)
     unsigned int spec_levels; // bit l: level l ran the fused filter (hit or miss)
     unsigned int spec_err;    // captured count != window total (internal consistency check)
-    int pad2_;
+    int dist_halt;            // sharded: 1 = survivors exceed the gather buffer (host adds levels), 2 = k >= N
     unsigned int seq;         // host mirror only: publish sequence number, written last
     int pad_seq;
     int tl_on;                // timeline mode (profile = 3): kernels stamp tl[]

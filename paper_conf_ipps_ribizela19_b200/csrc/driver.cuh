@@ -31,6 +31,7 @@
 
 #include "kernels.cuh"
 #include "quickselect.cuh"
+#include "comm.cuh"
 #include "sampleselect.h"
 
 using namespace ss;
@@ -117,6 +118,13 @@ struct ss_context {
     void* d_qsbuf[2] = {nullptr, nullptr};
     size_t cap_qsbuf = 0;
     cudaEvent_t ev_qs[2] = {nullptr, nullptr};
+    // ss_select_sharded: the communicator, the exchange buffers
+    // (sizes, per-rank counts, sample keys), the gather send/receive buffers
+    ss_comm::ShardComm* comm = nullptr;
+    void* d_dist = nullptr;
+    size_t cap_dist = 0;
+    void* d_gather[2] = {nullptr, nullptr};
+    size_t cap_gather[2] = {0, 0};
     int k2_occ[4][11] = {};          // count_kernel<T, H> resident CTAs per SM (per dtype, H)
     bool kw_attr[4][2] = {};         // window_kernel<T, APX> shared-memory attribute set
     bool host_timing = false;
@@ -509,6 +517,113 @@ ss_status launch_image(ss_context* c, int H, int lev, int s, int fixup, cudaStre
     return SS_OK;
 }
 
+// The exact chain of Fig. 1 (L95-127) from level lev0 to the plan's L: per
+// level K1 (sample + tree, or the base case), the fused window (planned spec
+// levels), K2 (count + K3/K4 tail) and K5 (filter), every kernel reading its
+// sizes from the device-resident LevelCtl of its level and exiting early once
+// the answer is known; then the final K1 (base case, or the "incomplete" flag
+// when an unlucky sample left more than B elements).  Level p.lev_first reads
+// `first_in`; level l > p.lev_first reads the buffer level l-1 wrote.
+struct ExactPlan {
+    int b0, bd, s, s_deep;
+    u32 B;
+    int L;                            // levels [.., L) are enqueued, then the final K1
+    bool spec_plan[SS_MAX_LEVELS];    // level l gets the fused window kernel
+    const void* sample0;              // sample keys of level lev_first gathered ahead (or NULL)
+    int lev_first;
+};
+
+template <typename T>
+ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first_in, int lev0, cudaStream_t q) {
+    typedef typename Traits<T>::Key K;
+    ss_status rc;
+    const T* in = lev0 > p.lev_first ? reinterpret_cast<const T*>(c->d_buf[(lev0 - 1) & 1]) : first_in;
+    int lev = lev0;
+    for (; lev < p.L; ++lev) {
+        const int b = lev ? p.bd : p.b0, H = log2i(b);
+        const u32 grid = grid_for<T>(c, H);
+        const int sl = lev && !p.spec_plan[lev] ? p.s_deep : p.s;
+        const int sl_next = lev + 1 < p.L && !p.spec_plan[lev + 1] ? p.s_deep : p.s;
+        K* pre_next = lev + 1 < p.L && sl_next <= WIDE_K1_MAX_S
+                          ? reinterpret_cast<K*>(c->d_presample) + (size_t)(lev + 1) * MAX_S : nullptr;
+        const void* pre_this = lev == p.lev_first ? p.sample0
+                                        : (p.spec_plan[lev - 1] ? (const void*)(reinterpret_cast<K*>(c->d_presample) +
+                                                                              (size_t)lev * MAX_S)
+                                                              : nullptr);
+        const bool wide = sl <= WIDE_K1_MAX_S;
+        CountArgs a{};
+        if (wide) a.image = c->d_image + (size_t)lev * K2_IMAGE_SLOT;
+        a.ctl = c->d_ctl + lev;
+        a.ctl_next = c->d_ctl + lev + 1;
+        a.res = c->d_res;
+        a.tree = reinterpret_cast<K*>(c->d_tree) + (size_t)lev * MAX_B;
+        a.spl = reinterpret_cast<K*>(c->d_spl) + (size_t)lev * MAX_B;
+        a.eq = c->d_eq + (size_t)lev * MAX_B;
+        a.oracles = c->d_oracles;
+        a.cta_counts = c->d_cta_counts;
+        a.totals = c->d_totals + (size_t)lev * MAX_B;
+        a.lut = c->cfg.classify == 0;
+        a.lut_stats = lev == 0 ? c->d_res->lut_stats : nullptr;
+        a.level = lev;
+        a.tail = TAIL_EXACT;
+        a.cap_out = c->d_buf[lev & 1];   // the fused filter's window copy = next level's input
+        if (wide) {
+            if ((rc = launch_k1_wide<T>(c, in, lev, sl, p.B, q, pre_this))) return rc;
+            if (p.spec_plan[lev]) {         // fused filter (streams iff the sample window speculates)
+                CountArgs w = a;
+                const SpecCfg sp = spec_params(c);
+                w.sorted = reinterpret_cast<K*>(c->d_sorted) + (size_t)lev * MAX_S;
+                w.s = sl;
+                w.spec_min_n = sp.min_n;
+                w.spec_z = sp.z;
+                w.spec_max_frac = sp.max_frac;
+                w.sample_next = pre_next;
+                w.s_next = sl_next;
+                w.seed = (u64)c->cfg.seed;
+                mark(c, lev, 1, 0, q);
+                if ((rc = launch_window<T>(c, H, in, w, q))) return rc;
+                mark(c, lev, 1, 1, q);        // slot (lev, K2) = the fused kernel on planned levels
+                ++c->launches;
+            }
+            if (lev == 0 || p.spec_plan[lev]) {
+                if ((rc = launch_image<T>(c, H, lev, sl, 1, q))) return rc;
+            } else {
+                // small deeper level: each count CTA builds the tree from
+                // the sorted sample itself and walks it (no image kernel,
+                // no lookup table)
+                a.image = nullptr;
+                a.sorted = reinterpret_cast<K*>(c->d_sorted) + (size_t)lev * MAX_S;
+                a.s = sl;
+                a.fixup = 1;
+                a.lut = 0;
+            }
+        } else if ((rc = launch_k1<T>(c, in, lev, sl, b, 1, p.B, 0, q))) {
+            return rc;
+        }
+        if (!(wide && p.spec_plan[lev])) mark(c, lev, 1, 0, q);
+        if ((rc = launch_count<T>(c, H, in, a, q))) return rc;
+        if (!(wide && p.spec_plan[lev])) mark(c, lev, 1, 1, q);
+        ++c->launches;
+        if (a.grid != grid) return fail(c, SS_ERR_INTERNAL, "grid mismatch");
+        T* out = reinterpret_cast<T*>(c->d_buf[lev & 1]);
+        FilterArgs f{};
+        f.ctl = c->d_ctl + lev;
+        f.res = c->d_res;
+        f.oracles = c->d_oracles;
+        f.cta_counts = c->d_cta_counts;
+        f.b_count = (u32)b;
+        f.grid = grid;
+        f.level = lev;
+        mark(c, lev, 2, 0, q);
+        CK(launch_pdl(filter_kernel<T>, dim3(grid), dim3(K5_THREADS), FILTER_SMEM, q, in, out, f));
+        CKLAUNCH("filter_kernel");
+        mark(c, lev, 2, 1, q);
+        ++c->launches;
+        in = out;
+    }
+    return launch_k1<T>(c, in, lev, lev ? p.s_deep : p.s, lev ? p.bd : p.b0, 1, p.B, 1, q);
+}
+
 template <typename T>
 ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cudaStream_t st) {
     typedef typename Traits<T>::Key K;
@@ -546,94 +661,14 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
         ++c->launches;
         return SS_OK;
     };
-    // levels [lev0, L) and the final K1 (base case or "incomplete" flag)
+    ExactPlan plan{};
+    plan.b0 = b0; plan.bd = bd; plan.s = s; plan.s_deep = s_deep; plan.B = B; plan.L = L;
+    std::copy(spec_plan, spec_plan + SS_MAX_LEVELS, plan.spec_plan);
+    plan.sample0 = sample0;
+    plan.lev_first = 0;
     auto enqueue_levels = [&](int lev0, cudaStream_t q) -> ss_status {
-        ss_status rc2;
-        const T* in = lev0 ? reinterpret_cast<const T*>(c->d_buf[(lev0 - 1) & 1]) : d;
-        int lev = lev0;
-        for (; lev < L; ++lev) {
-            const int b = lev ? bd : b0, H = log2i(b);
-            const u32 grid = grid_for<T>(c, H);
-            const int sl = lev && !spec_plan[lev] ? s_deep : s;
-            const int sl_next = lev + 1 < L && !spec_plan[lev + 1] ? s_deep : s;
-            K* pre_next = lev + 1 < L && sl_next <= WIDE_K1_MAX_S
-                              ? reinterpret_cast<K*>(c->d_presample) + (size_t)(lev + 1) * MAX_S : nullptr;
-            const void* pre_this = lev == 0 ? (const void*)sample0
-                                            : (spec_plan[lev - 1] ? (const void*)(reinterpret_cast<K*>(c->d_presample) +
-                                                                                  (size_t)lev * MAX_S)
-                                                                  : nullptr);
-            const bool wide = sl <= WIDE_K1_MAX_S;
-            CountArgs a{};
-            if (wide) a.image = c->d_image + (size_t)lev * K2_IMAGE_SLOT;
-            a.ctl = c->d_ctl + lev;
-            a.ctl_next = c->d_ctl + lev + 1;
-            a.res = c->d_res;
-            a.tree = reinterpret_cast<K*>(c->d_tree) + (size_t)lev * MAX_B;
-            a.spl = reinterpret_cast<K*>(c->d_spl) + (size_t)lev * MAX_B;
-            a.eq = c->d_eq + (size_t)lev * MAX_B;
-            a.oracles = c->d_oracles;
-            a.cta_counts = c->d_cta_counts;
-            a.totals = c->d_totals + (size_t)lev * MAX_B;
-            a.lut = c->cfg.classify == 0;
-            a.lut_stats = lev == 0 ? c->d_res->lut_stats : nullptr;
-            a.level = lev;
-            a.tail = TAIL_EXACT;
-            a.cap_out = c->d_buf[lev & 1];   // the fused filter's window copy = next level's input
-            if (wide) {
-                if ((rc2 = launch_k1_wide<T>(c, in, lev, sl, B, q, pre_this))) return rc2;
-                if (spec_plan[lev]) {         // fused filter (streams iff the sample window speculates)
-                    CountArgs w = a;
-                    const SpecCfg sp = spec_params(c);
-                    w.sorted = reinterpret_cast<K*>(c->d_sorted) + (size_t)lev * MAX_S;
-                    w.s = sl;
-                    w.spec_min_n = sp.min_n;
-                    w.spec_z = sp.z;
-                    w.spec_max_frac = sp.max_frac;
-                    w.sample_next = pre_next;
-                    w.s_next = sl_next;
-                    w.seed = (u64)c->cfg.seed;
-                    mark(c, lev, 1, 0, q);
-                    if ((rc2 = launch_window<T>(c, H, in, w, q))) return rc2;
-                    mark(c, lev, 1, 1, q);        // slot (lev, K2) = the fused kernel on planned levels
-                    ++c->launches;
-                }
-                if (lev == 0 || spec_plan[lev]) {
-                    if ((rc2 = launch_image<T>(c, H, lev, sl, 1, q))) return rc2;
-                } else {
-                    // small deeper level: each count CTA builds the tree from
-                    // the sorted sample itself and walks it (no image kernel,
-                    // no lookup table)
-                    a.image = nullptr;
-                    a.sorted = reinterpret_cast<K*>(c->d_sorted) + (size_t)lev * MAX_S;
-                    a.s = sl;
-                    a.fixup = 1;
-                    a.lut = 0;
-                }
-            } else if ((rc2 = launch_k1<T>(c, in, lev, sl, b, 1, B, 0, q))) {
-                return rc2;
-            }
-            if (!(wide && spec_plan[lev])) mark(c, lev, 1, 0, q);
-            if ((rc2 = launch_count<T>(c, H, in, a, q))) return rc2;
-            if (!(wide && spec_plan[lev])) mark(c, lev, 1, 1, q);
-            ++c->launches;
-            if (a.grid != grid) return fail(c, SS_ERR_INTERNAL, "grid mismatch");
-            T* out = reinterpret_cast<T*>(c->d_buf[lev & 1]);
-            FilterArgs f{};
-            f.ctl = c->d_ctl + lev;
-            f.res = c->d_res;
-            f.oracles = c->d_oracles;
-            f.cta_counts = c->d_cta_counts;
-            f.b_count = (u32)b;
-            f.grid = grid;
-            f.level = lev;
-            mark(c, lev, 2, 0, q);
-            CK(launch_pdl(filter_kernel<T>, dim3(grid), dim3(K5_THREADS), FILTER_SMEM, q, in, out, f));
-            CKLAUNCH("filter_kernel");
-            mark(c, lev, 2, 1, q);
-            ++c->launches;
-            in = out;
-        }
-        return launch_k1<T>(c, in, lev, lev ? s_deep : s, lev ? bd : b0, 1, B, 1, q);
+        plan.L = L;
+        return enqueue_exact_levels<T>(c, plan, d, lev0, q);
     };
     // the planned part of the call: one CUDA graph launch (events of
     // profile 1/2 cannot live in a graph: those calls launch directly)
@@ -743,7 +778,9 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     if (c->host_timing) c->ht[2] += now_us() - t_w;
     const double t_s = c->host_timing ? now_us() : 0.0;
     // rare: an unlucky sample left more than B elements after the planned levels
+    int extra_rounds = 0;
     while (!c->h_res->done) {
+        ++extra_rounds;
         if (!c->h_res->incomplete || L >= SS_MAX_LEVELS - 2)
             return fail(c, SS_ERR_INTERNAL, "recursion did not terminate");
         CK(cudaMemsetAsync(&c->d_res->incomplete, 0, sizeof(int), st));
@@ -764,6 +801,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     S.lut_marker = (int32_t)r.lut_stats[1];
     S.spec_levels = (int32_t)r.spec_levels;
     S.fused_levels = (int32_t)r.fused_levels;
+    S.incomplete_rounds = extra_rounds;
     if (r.spec_err) return fail(c, SS_ERR_INTERNAL, "fused filter: captured count != window total");
     double bytes = 0;
     const double Sz = (double)sizeof(T);
@@ -1193,6 +1231,8 @@ ss_status run_quick(ss_context* c, const T* d, u64 n, u64 k, void* h_result, int
 }
 
 
+
+#include "sharded.cuh"
 
 }  // namespace
 

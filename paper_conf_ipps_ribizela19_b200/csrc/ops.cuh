@@ -23,7 +23,8 @@
     ss_status op_step_filter(ss_context* c, const T* d, ss::u64 n, const uint8_t* oracles, int bucket,        \
                              T* out, ss::u64* count, cudaStream_t st);                                        \
     ss_status op_keys_to_values(ss_context* c, const T* tag, const void* keys, ss::u64 count, void* values,   \
-                                cudaStream_t st);
+                                cudaStream_t st);                                                             \
+    ss_status op_sharded(ss_context* c, const T* d, ss::u64 n_local, ss::u64 k, void* h_result, cudaStream_t st);
 
 SS_OPS_DECL(float)
 SS_OPS_DECL(double)
@@ -111,5 +112,8 @@ ss_status op_keys_to_values(ss_context* c, const InstT*, const void* keys, u64 c
     keys_to_values_kernel<InstT><<<blocks, 256, 0, st>>>((const K*)keys, count, (K*)values);
     CKLAUNCH("keys_to_values_kernel");
     return SS_OK;
+}
+ss_status op_sharded(ss_context* c, const InstT* d, u64 n_local, u64 k, void* h_result, cudaStream_t st) {
+    return run_sharded<InstT>(c, d, n_local, k, h_result, st);
 }
 #endif  // SS_INST_T

@@ -1,19 +1,27 @@
-"""Multi-process (world_size 2, gloo, CPU) tests of the sharded driver's host
-protocol: proportional sample slots, sample all-gather, count all-reduce,
-global bucket search, equality exit, survivor gather.  The per-rank steps are
-the CPU oracle's (tests/_oracle_steps.py)."""
+"""Multi-process (world_size 2, gloo, CPU) tests of the sharded protocol and
+its host plumbing.
+
+* The protocol of ss_select_sharded (csrc/sharded.cuh) replayed by the CPU
+  model tests/_sharded_model.py over real gloo collectives: proportional
+  sample slots, the disjoint-slot sum exchanges (sample, per-rank counts,
+  gather), the window hit / equality exit / directed miss decision -- every
+  rank must take the same decisions and return the oracle's answer, for iid,
+  non-iid, empty, all-equal, few-distinct and integer shards.
+* The communicator plumbing of paper_conf_ipps_ribizela19_b200.sharded: a
+  NCCL unique id drawn on rank 0 reaches every rank intact through
+  torch.distributed (the part of comm_init_from_process_group that needs no
+  GPU)."""
 import os
 import socket
 
 import numpy as np
 import pytest
-import torch
 import torch.distributed as dist
 import torch.multiprocessing as mp
 
 import datagen
 import oracle
-from paper_conf_ipps_ribizela19_b200.sharded import ShardedSelect, TorchDistComm
+from _sharded_model import ShardedModel, TorchDistExchange, slot_range
 
 WORLD = 2
 
@@ -40,21 +48,34 @@ def _shards(case):
     raise ValueError(case)
 
 
-def _worker(rank, port, case, ks, thresholds, q):
+def _worker(rank, port, case, ks, gathers, q):
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=WORLD)
     try:
-        from _oracle_steps import OracleSteps
-        shard = torch.from_numpy(_shards(case)[rank])
+        shard = _shards(case)[rank]
         res = []
-        for thr in thresholds:
-            sel = ShardedSelect(OracleSteps(), TorchDistComm(), b=16, s=256, gather_threshold=thr)
+        for G in gathers:
+            m = ShardedModel(TorchDistExchange(), s=256, gather=G)
             for k in ks:
-                v = sel.select(shard, k)
-                res.append((thr, k, np.asarray(v).tobytes(), list(sel.last_levels)))
+                v = m.select(shard, k)
+                res.append((G, k, np.asarray(v).tobytes(), list(m.levels), list(m.hits)))
         q.put((rank, res))
     finally:
         dist.destroy_process_group()
+
+
+def _run(target, args):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=target, args=(r, port, *args, q)) for r in range(WORLD)]
+    for p in procs:
+        p.start()
+    out = dict(q.get(timeout=300) for _ in procs)
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    return out
 
 
 @pytest.mark.parametrize("case", ["iid", "noniid", "empty", "equal", "distinct", "int"])
@@ -62,29 +83,49 @@ def test_sharded_protocol_gloo(case):
     full = np.concatenate(_shards(case))
     N = full.size
     ks = sorted({0, 1, N // 2, N - 1, datagen.rank(N, 4)})
-    thresholds = [0, 64, 1 << 30]           # all levels distributed / mixed / gather at once
-    ctx = mp.get_context("spawn")
-    q = ctx.Queue()
-    port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, port, case, ks, thresholds, q)) for r in range(WORLD)]
-    for p in procs:
-        p.start()
-    out = dict(q.get(timeout=300) for _ in procs)
-    for p in procs:
-        p.join(timeout=60)
-        assert p.exitcode == 0
-    assert out[0] == out[1]                 # every rank returns the identical answer
-    for thr, k, bits, levels in out[0]:
-        assert bits == np.asarray(oracle.select(full, k)).tobytes(), (case, thr, k)
-        assert all(a > b for a, b in zip(levels, levels[1:]))
-        if thr == 0 and case not in ("equal", "distinct"):
-            assert len(levels) >= 1
+    gathers = [16, 512, 1 << 30]            # several sharded levels / one / gather at once
+    out = _run(_worker, (case, ks, gathers))
+    assert out[0] == out[1]                 # every rank takes the same decisions and answer
+    for G, k, bits, levels, hits in out[0]:
+        assert bits == np.asarray(oracle.select(full, k)).tobytes(), (case, G, k)
+        for i in range(len(levels) - 1):     # a hit shrinks the level; a miss re-streams it
+            assert levels[i + 1] < levels[i] if hits[i] else levels[i + 1] == levels[i], (levels, hits)
+        for i in range(len(hits) - 1):       # the directed level after a miss always holds k
+            assert hits[i] or hits[i + 1], hits
+        if G == 16 and case in ("iid", "noniid", "int"):
+            assert len(levels) >= 2
+
+
+def _uid_worker(rank, port, q):
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=WORLD)
+    try:
+        import paper_conf_ipps_ribizela19_b200 as ss
+        try:
+            uid = ss.nccl_unique_id() if rank == 0 else None
+        except ss.SSError as e:      # NCCL not loadable here: report, the test skips
+            uid = ("unavailable", str(e))
+        obj = [uid]
+        dist.broadcast_object_list(obj, src=0)
+        q.put((rank, obj[0]))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_nccl_unique_id_broadcast_gloo():
+    from paper_conf_ipps_ribizela19_b200 import build
+    build.build()
+    out = _run(_uid_worker, ())
+    if isinstance(out[0], tuple):
+        pytest.skip(f"NCCL unavailable: {out[0][1]}")
+    assert isinstance(out[0], bytes) and len(out[0]) == 128
+    assert out[0] == out[1]
 
 
 def test_slot_ranges_partition_the_sample():
     sizes = [5, 0, 17, 3, 1000]
     s = 4096
-    ranges = [ShardedSelect.slot_range(sizes, r, s) for r in range(len(sizes))]
+    ranges = [slot_range(sizes, r, s) for r in range(len(sizes))]
     assert ranges[0][0] == 0 and ranges[-1][1] == s
     for (a0, a1), (b0, b1) in zip(ranges, ranges[1:]):
         assert a1 == b0
