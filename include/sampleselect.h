@@ -75,16 +75,18 @@ typedef struct {
                              marker cells are light, else the Fig. 4 tree walk);
                              1 = always the tree walk.  Same buckets either way. default 0 */
     uint64_t seed;        /* sampling seed (reading R7). default 0x5A17 */
-    int32_t fused_filter; /* exact levels: 1 = (default) fused speculative filter on levels with
-                             n_l >= spec_min_n: the sample predicts a window of buckets around
-                             rank k and the count kernel copies the window's elements to the
-                             next level while it counts (no oracle bytes, no filter pass; a
-                             miss falls back to a re-classifying filter); 0 = always the
-                             paper's oracle bytes + filter kernel (§IV.B-c).  Same answer. */
+    int32_t fused_filter; /* exact levels: 1 = (default) fused levels where n_l >= spec_min_n:
+                             the level's sample (16384 keys, or sample_size) gives a key
+                             window around rank k (two order statistics, no sort) and one
+                             pass counts the keys below it and copies the keys inside it to
+                             the next level (reading R21: a SampleSelect level with two
+                             splitters, no oracle bytes, no filter pass; a miss re-runs the
+                             level with the paper's tree); 0 = always the paper's level:
+                             b-bucket tree, oracle bytes, filter kernel (§IV.B).  Same answer. */
     float spec_z;         /* window half-width in standard deviations of the sample rank of k
-                             (Binomial(s, k/n)); default 3 (miss probability ~3e-3; a miss
-                             re-runs the level with the paper's filter) */
-    int64_t spec_min_n;   /* levels with at least this many elements speculate. default 2^22 */
+                             (Binomial(s, k/n)); default 3 (miss probability ~3e-3 per level) */
+    int64_t spec_min_n;   /* levels with at least this many elements (host estimate) are fused
+                             levels. default 2^16 */
     float spec_max_frac;  /* speculate only if the window holds at most this fraction of the
                              sample. default 0.25 */
     int32_t shard_gather_log2; /* ss_select_sharded: survivors are gathered onto every rank once

@@ -76,7 +76,7 @@ ss_status ss_create(int device, ss_context** out) {
     c->cfg.classify = 0;
     c->cfg.fused_filter = 1;
     c->cfg.spec_z = 3.0f;
-    c->cfg.spec_min_n = (int64_t)1 << 22;
+    c->cfg.spec_min_n = (int64_t)1 << 16;
     c->cfg.spec_max_frac = 0.25f;
     c->cfg.shard_gather_log2 = 0;
     DevGuard g(device);
@@ -494,6 +494,7 @@ ss_status ss_comm_init(ss_context* c, const char id[128], int nranks, int rank) 
     if (!comm) return fail(c, rc, err);
     delete c->comm;
     c->comm = comm;
+    c->dist_n_plan = 0;
     return SS_OK;
 }
 
@@ -509,6 +510,7 @@ ss_status ss_comm_init_local(ss_context* c, ss_local_group* g, int rank) {
     if (!comm) return fail(c, rc, err);
     delete c->comm;
     c->comm = comm;
+    c->dist_n_plan = 0;
     return SS_OK;
 }
 

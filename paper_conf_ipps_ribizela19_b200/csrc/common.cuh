@@ -88,6 +88,8 @@ struct LevelCtl {
     u32 directed;   // the window is [klo, klo + kspan) from the previous level's miss, not the sample
     float dfrac;    // directed window: expected fraction of the level inside it
     u32 pad3_;
+    const void* src;// level 0: the call's input (written by the init kernel, whose argument is patched
+                    // per call in a cached CUDA graph); NULL on deeper levels
 };
 
 struct SelectResult {
@@ -106,7 +108,9 @@ struct SelectResult {
     unsigned int spec_err;    // captured count != window total (internal consistency check)
     int dist_halt;            // sharded: 1 = survivors exceed the gather buffer (host adds levels), 2 = k >= N
     unsigned int seq;         // host mirror only: publish sequence number, written last
-    int pad_seq;
+    int halt;                 // level + 1 of a fused level whose window missed rank k (or could not
+                              // shrink the level): the chain stopped (done), the host re-runs it
+    unsigned long long dist_n;// sharded: the size of the union of the shards (the host plans the next call with it)
     int tl_on;                // timeline mode (profile = 3): kernels stamp tl[]
     int pad_;
     u64 t_init;               // %globaltimer at the init kernel (timeline origin)

@@ -44,6 +44,7 @@ static __global__ void dist_check_kernel(const u64* __restrict__ sizes, int P, u
     if (threadIdx.x != 0) return;
     u64 N = 0;
     for (int q = 0; q < P; ++q) N += sizes[q];
+    res->dist_n = N;
     if (k >= N) {
         res->dist_halt = 2;
         res->done = 1;

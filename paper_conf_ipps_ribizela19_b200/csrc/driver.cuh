@@ -64,11 +64,11 @@ struct ss_context {
     u32 seq = 0;                     // publishes issued (host count, lockstep with *d_seq)
     u32* d_seq = nullptr;            // device publish counter
     // CUDA graphs of whole calls (init + levels + final K1 + publish), one per
-    // (dtype, input, n, plan); the rank k is patched into the init node
+    // (dtype, n, plan); the rank k and the input pointer are patched into the
+    // init node (level 0's kernels read the input from LevelCtl::src)
     struct GraphEntry {
         bool used = false;
         int dt = -1;
-        const void* ptr = nullptr;
         u64 n = 0;
         int b0 = 0, bd = 0, s = 0, sd = 0, L = 0, prof = 0;
         u32 B = 0;
@@ -80,6 +80,7 @@ struct ss_context {
         void* init_args[16] = {};
         unsigned char init_store[256] = {};   // backing store of the init kernel's arguments
         size_t k_offset = 0;                  // where k lives in init_store
+        size_t d_offset = 0;                  // where the input pointer lives in init_store
         int kernels = 0;
         u64 stamp = 0;
     } graphs[8];
@@ -121,6 +122,7 @@ struct ss_context {
     // ss_select_sharded: the communicator, the exchange buffers
     // (sizes, per-rank counts, sample keys), the gather send/receive buffers
     ss_comm::ShardComm* comm = nullptr;
+    u64 dist_n_plan = 0;             // size of the union seen by the last sharded call (0: exchange first)
     void* d_dist = nullptr;
     size_t cap_dist = 0;
     void* d_gather[2] = {nullptr, nullptr};
@@ -434,24 +436,33 @@ SpecCfg spec_params(const ss_context* c) {
     return p;
 }
 
-int expected_levels(const ss_context* c, u64 n, int b0, int bd, int s0, int sd, u32 B, bool* spec_plan) {
-    // n_{l+1} ~ n_l / b_l times the size bias of the bucket holding k (~1.1
-    // for s/b = 16); plan with 1.5x slack, fall back to more levels if needed.
-    // A fused-filter level keeps its window: at most (2 (z sigma + 2) + 1) / s
-    // of the level with sigma <= sqrt(s) / 2, plus one bucket at each end.
+// Fused-level sample sizes (K1w): the configured sample_size if set (at least
+// 1024), else 16384 -- the window is ~6 z / sqrt(s) of the level.
+inline int fused_sample(const ss_config& cfg) {
+    if (cfg.sample_size > 0) return std::max(1024, std::min(cfg.sample_size, 16384));
+    return 16384;
+}
+
+inline double window_frac(float z, int s) {
+    return (2.0 * (z * 0.5 * std::sqrt((double)s) + 2.0) + 1.0) / s;
+}
+
+// The planned levels of an exact call.  A paper level keeps ~1.5 / b of its
+// input (the bucket holding k is size-biased, ~1.1 for s / b = 16; 1.5 is
+// slack); a fused level keeps its window (<= window_frac of it, plus chunk
+// padding).  Levels with at least spec_min_n elements (host estimate) are
+// fused when fused_filter is on.  An under-estimate is caught on the device
+// (the final K1 flags "incomplete") and more levels are enqueued.
+int expected_levels(const ss_context* c, u64 n, int b0, int bd, int sf0, int sfd, u32 B, bool* spec_plan) {
     const SpecCfg sp = spec_params(c);
     int L = 0;
     double m = (double)n;
     while (m > (double)B && L < SS_MAX_LEVELS - 2) {
-        // levels whose size may reach min_n get the fused-filter kernel
-        // enqueued (it exits unless the device-side window decision is
-        // "spec") and draw the level-0 sample size s0 (a narrower window)
-        const bool cand = s0 <= WIDE_K1_MAX_S && 2.0 * m >= (double)sp.min_n && sp.min_n != ~0ull;
-        const int b = L ? bd : b0, s = L && !cand ? sd : s0;
-        const double f = (2.0 * (sp.z * 0.5 * std::sqrt((double)s) + 2.0) + 1.0) / s;
-        const bool spec = cand && m >= (double)sp.min_n && f <= sp.max_frac;
-        if (spec_plan) spec_plan[L] = cand && f <= sp.max_frac;
-        m = spec ? m * 1.2 * f : m * 1.5 / b;
+        const int b = L ? bd : b0;
+        const double f = window_frac(sp.z, L ? sfd : sf0);
+        const bool spec = sp.min_n != ~0ull && m >= (double)sp.min_n && f <= sp.max_frac;
+        if (spec_plan) spec_plan[L] = spec;
+        m = spec ? m * 1.2 * f + (double)c->sms * 32.0 : m * 1.5 / b;
         ++L;
     }
     return L;
@@ -517,21 +528,53 @@ ss_status launch_image(ss_context* c, int H, int lev, int s, int fixup, cudaStre
     return SS_OK;
 }
 
-// The exact chain of Fig. 1 (L95-127) from level lev0 to the plan's L: per
-// level K1 (sample + tree, or the base case), the fused window (planned spec
-// levels), K2 (count + K3/K4 tail) and K5 (filter), every kernel reading its
-// sizes from the device-resident LevelCtl of its level and exiting early once
-// the answer is known; then the final K1 (base case, or the "incomplete" flag
-// when an unlucky sample left more than B elements).  Level p.lev_first reads
-// `first_in`; level l > p.lev_first reads the buffer level l-1 wrote.
+// The exact chain of Fig. 1 (L95-127) from level lev0 to the plan's L.  A
+// paper level is K1 (sample + sort, or the base case), the tree image, K2
+// (count + K3/K4 tail) and K5 (filter); a fused level (spec_plan) is K1w (the
+// window straight from the sample, window_select_kernel) and the fused
+// count + filter pass (window_kernel) -- nothing else is enqueued behind it:
+// a miss halts the chain (SelectResult::halt) and the host re-runs that level
+// the paper's way.  Every kernel reads its sizes from the device-resident
+// LevelCtl of its level and exits early once the answer is known; the chain
+// ends with the final K1 (base case, or the "incomplete" flag when an unlucky
+// sample left more than B elements).  Level p.lev_first reads `first_in`;
+// level l > p.lev_first reads the buffer level l-1 wrote (d_buf[(l-1) & 1]).
 struct ExactPlan {
     int b0, bd, s, s_deep;
+    int sf0, sfd;                     // sample sizes of fused levels: level 0, deeper levels
     u32 B;
     int L;                            // levels [.., L) are enqueued, then the final K1
-    bool spec_plan[SS_MAX_LEVELS];    // level l gets the fused window kernel
+    bool spec_plan[SS_MAX_LEVELS];    // level l is a fused level
     const void* sample0;              // sample keys of level lev_first gathered ahead (or NULL)
     int lev_first;
 };
+
+inline int plan_sample(const ExactPlan& p, int lev) {
+    if (p.spec_plan[lev]) return lev ? p.sfd : p.sf0;
+    return lev ? p.s_deep : p.s;
+}
+
+template <typename T>
+ss_status launch_wsel(ss_context* c, const T* in, int lev, int s, u32 B, const void* pre, cudaStream_t q) {
+    typedef typename Traits<T>::Key K;
+    const SpecCfg sp = spec_params(c);
+    mark(c, lev, 0, 0, q);
+#define SS_WSEL_CASE(E)                                                                                    \
+    case E:                                                                                                \
+        CK(launch_pdl(window_select_kernel<T, E>, dim3(1), dim3(WS_THREADS), 0, q, in, c->d_ctl + lev,     \
+                      c->d_ctl + lev + 1, c->d_res, reinterpret_cast<const K*>(pre), B, (u64)c->cfg.seed, \
+                      lev, sp.z, sp.max_frac));                                                            \
+        break;
+    switch (s / WS_THREADS) {
+        SS_WSEL_CASE(1) SS_WSEL_CASE(2) SS_WSEL_CASE(4) SS_WSEL_CASE(8) SS_WSEL_CASE(16)
+    default: return fail(c, SS_ERR_INTERNAL, "fused-level sample size must be 1024 * 2^i <= 16384");
+    }
+#undef SS_WSEL_CASE
+    CKLAUNCH("window_select_kernel");
+    mark(c, lev, 0, 1, q);
+    ++c->launches;
+    return SS_OK;
+}
 
 template <typename T>
 ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first_in, int lev0, cudaStream_t q) {
@@ -541,15 +584,40 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
     int lev = lev0;
     for (; lev < p.L; ++lev) {
         const int b = lev ? p.bd : p.b0, H = log2i(b);
-        const u32 grid = grid_for<T>(c, H);
-        const int sl = lev && !p.spec_plan[lev] ? p.s_deep : p.s;
-        const int sl_next = lev + 1 < p.L && !p.spec_plan[lev + 1] ? p.s_deep : p.s;
-        K* pre_next = lev + 1 < p.L && sl_next <= WIDE_K1_MAX_S
+        const int sl = plan_sample(p, lev);
+        const int sl_next = lev + 1 < p.L ? plan_sample(p, lev + 1) : 0;
+        // a fused level's tail gathers the next level's sample from its output
+        K* pre_next = lev + 1 < p.L && (p.spec_plan[lev + 1] || sl_next <= WIDE_K1_MAX_S)
                           ? reinterpret_cast<K*>(c->d_presample) + (size_t)(lev + 1) * MAX_S : nullptr;
         const void* pre_this = lev == p.lev_first ? p.sample0
-                                        : (p.spec_plan[lev - 1] ? (const void*)(reinterpret_cast<K*>(c->d_presample) +
-                                                                              (size_t)lev * MAX_S)
-                                                              : nullptr);
+                               : (lev > 0 && p.spec_plan[lev - 1]
+                                      ? (const void*)(reinterpret_cast<K*>(c->d_presample) + (size_t)lev * MAX_S)
+                                      : nullptr);
+        if (p.spec_plan[lev]) {               // fused level: K1w + count/filter in one pass
+            if ((rc = launch_wsel<T>(c, in, lev, sl, p.B, pre_this, q))) return rc;
+            const SpecCfg sp = spec_params(c);
+            CountArgs w{};
+            w.ctl = c->d_ctl + lev;
+            w.ctl_next = c->d_ctl + lev + 1;
+            w.res = c->d_res;
+            w.level = lev;
+            w.tail = TAIL_EXACT;
+            w.cap_out = c->d_buf[lev & 1];    // the window = the next level's input
+            w.spec_min_n = sp.min_n;
+            w.spec_z = sp.z;
+            w.spec_max_frac = sp.max_frac;
+            w.sample_next = pre_next;
+            w.s_next = sl_next;
+            w.seed = (u64)c->cfg.seed;
+            w.halt_on_miss = 1;
+            mark(c, lev, 1, 0, q);
+            if ((rc = launch_window<T>(c, H, in, w, q))) return rc;
+            mark(c, lev, 1, 1, q);
+            ++c->launches;
+            in = reinterpret_cast<const T*>(c->d_buf[lev & 1]);
+            continue;
+        }
+        const u32 grid = grid_for<T>(c, H);
         const bool wide = sl <= WIDE_K1_MAX_S;
         CountArgs a{};
         if (wide) a.image = c->d_image + (size_t)lev * K2_IMAGE_SLOT;
@@ -566,26 +634,9 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
         a.lut_stats = lev == 0 ? c->d_res->lut_stats : nullptr;
         a.level = lev;
         a.tail = TAIL_EXACT;
-        a.cap_out = c->d_buf[lev & 1];   // the fused filter's window copy = next level's input
         if (wide) {
             if ((rc = launch_k1_wide<T>(c, in, lev, sl, p.B, q, pre_this))) return rc;
-            if (p.spec_plan[lev]) {         // fused filter (streams iff the sample window speculates)
-                CountArgs w = a;
-                const SpecCfg sp = spec_params(c);
-                w.sorted = reinterpret_cast<K*>(c->d_sorted) + (size_t)lev * MAX_S;
-                w.s = sl;
-                w.spec_min_n = sp.min_n;
-                w.spec_z = sp.z;
-                w.spec_max_frac = sp.max_frac;
-                w.sample_next = pre_next;
-                w.s_next = sl_next;
-                w.seed = (u64)c->cfg.seed;
-                mark(c, lev, 1, 0, q);
-                if ((rc = launch_window<T>(c, H, in, w, q))) return rc;
-                mark(c, lev, 1, 1, q);        // slot (lev, K2) = the fused kernel on planned levels
-                ++c->launches;
-            }
-            if (lev == 0 || p.spec_plan[lev]) {
+            if (lev == 0) {
                 if ((rc = launch_image<T>(c, H, lev, sl, 1, q))) return rc;
             } else {
                 // small deeper level: each count CTA builds the tree from
@@ -600,9 +651,9 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
         } else if ((rc = launch_k1<T>(c, in, lev, sl, b, 1, p.B, 0, q))) {
             return rc;
         }
-        if (!(wide && p.spec_plan[lev])) mark(c, lev, 1, 0, q);
+        mark(c, lev, 1, 0, q);
         if ((rc = launch_count<T>(c, H, in, a, q))) return rc;
-        if (!(wide && p.spec_plan[lev])) mark(c, lev, 1, 1, q);
+        mark(c, lev, 1, 1, q);
         ++c->launches;
         if (a.grid != grid) return fail(c, SS_ERR_INTERNAL, "grid mismatch");
         T* out = reinterpret_cast<T*>(c->d_buf[lev & 1]);
@@ -646,23 +697,27 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     for (int i = 0; i < 2; ++i)
         if ((rc = grow(c, &c->d_buf[i], &c->cap_buf[i], n * sizeof(T)))) return rc;
     bool spec_plan[SS_MAX_LEVELS] = {};
-    int L = expected_levels(c, n, b0, bd, s, s_deep, B, spec_plan);
-    // level 0's sample is gathered by the init kernel when the wide K1 ranks it
-    const bool pre0 = L > 0 && s <= WIDE_K1_MAX_S;
+    const int sf = fused_sample(c->cfg);
+    int L = expected_levels(c, n, b0, bd, sf, sf, B, spec_plan);
+    // level 0's sample is gathered by the init kernel (spread over the grid)
+    // when K1w or the wide K1 takes it from memory
+    const int s_init = L > 0 && spec_plan[0] ? sf : s;
+    const bool pre0 = L > 0 && (spec_plan[0] || s <= WIDE_K1_MAX_S);
     K* sample0 = pre0 ? reinterpret_cast<K*>(c->d_sample0) : nullptr;
     const int tl_on = c->cfg.profile == 3;
     // totals of every planned level are zeroed by init; levels beyond the plan
     // (the rare "incomplete" fallback) are zeroed before they run
     auto enqueue_init = [&](cudaStream_t q) -> ss_status {
-        CK(launch_pdl(init_kernel<T>, dim3(pre0 ? ((u32)s + 255u) / 256u : 1u), dim3(256), 0, q, c->d_ctl,
-                      (int)(SS_MAX_LEVELS + 1), c->d_totals, (int)((L + 1) * MAX_B), c->d_res, n, k, tl_on, d, s,
-                      (u64)c->cfg.seed, sample0));
+        CK(launch_pdl(init_kernel<T>, dim3(pre0 ? ((u32)s_init + 255u) / 256u : 1u), dim3(256), 0, q, c->d_ctl,
+                      (int)(SS_MAX_LEVELS + 1), c->d_totals, (int)((L + 1) * MAX_B), c->d_res, n, k, tl_on, d,
+                      s_init, (u64)c->cfg.seed, sample0));
         CKLAUNCH("init_kernel");
         ++c->launches;
         return SS_OK;
     };
     ExactPlan plan{};
     plan.b0 = b0; plan.bd = bd; plan.s = s; plan.s_deep = s_deep; plan.B = B; plan.L = L;
+    plan.sf0 = sf; plan.sfd = sf;
     std::copy(spec_plan, spec_plan + SS_MAX_LEVELS, plan.spec_plan);
     plan.sample0 = sample0;
     plan.lev_first = 0;
@@ -676,7 +731,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     ss_context::GraphEntry* ge = nullptr;
     if (graph) {
         for (auto& e : c->graphs)
-            if (e.used && e.dt == dt_code<T>() && e.ptr == d &&
+            if (e.used && e.dt == dt_code<T>() &&
                 e.n == n && e.b0 == b0 && e.bd == bd && e.s == s && e.sd == s_deep && e.L == L &&
                 e.prof == tl_on && e.B == B && e.seed == c->cfg.seed)
                 ge = &e;
@@ -732,7 +787,6 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             }
             slot->used = true;
             slot->dt = dt_code<T>();
-            slot->ptr = d;
             slot->n = n;
             slot->b0 = b0; slot->bd = bd; slot->s = s; slot->sd = s_deep; slot->L = L;
             slot->prof = tl_on; slot->B = B; slot->seed = c->cfg.seed;
@@ -750,6 +804,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
                 std::memcpy(slot->init_store + off, ip.kernelParams[i], sizes[i]);
                 slot->init_args[i] = slot->init_store + off;
                 if (i == 6) slot->k_offset = off;
+                if (i == 8) slot->d_offset = off;
                 off += sizes[i];
             }
             slot->init_params.kernelParams = slot->init_args;
@@ -758,8 +813,13 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             ge = slot;
             c->launches = launches0;
         } else {
+            // the rank and the input pointer are arguments of the init kernel
+            // only (later kernels read level 0's input from LevelCtl::src):
+            // patch them into the cached graph
             u64 kk = k;
+            const T* dd = d;
             std::memcpy(ge->init_store + ge->k_offset, &kk, sizeof(u64));
+            std::memcpy(ge->init_store + ge->d_offset, &dd, sizeof(const T*));
             CK(cudaGraphExecKernelNodeSetParams(ge->exec, ge->init_node, &ge->init_params));
         }
         ge->stamp = ++c->graph_clock;
@@ -777,17 +837,46 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     if ((rc = wait_publish(c, st))) return rc;
     if (c->host_timing) c->ht[2] += now_us() - t_w;
     const double t_s = c->host_timing ? now_us() : 0.0;
-    // rare: an unlucky sample left more than B elements after the planned levels
+    // rare: a fused level's window missed rank k (halt), or an unlucky sample
+    // left more than B elements after the planned levels (incomplete)
     int extra_rounds = 0;
-    while (!c->h_res->done) {
-        ++extra_rounds;
-        if (!c->h_res->incomplete || L >= SS_MAX_LEVELS - 2)
-            return fail(c, SS_ERR_INTERNAL, "recursion did not terminate");
-        CK(cudaMemsetAsync(&c->d_res->incomplete, 0, sizeof(int), st));
-        CK(cudaMemsetAsync(c->d_totals + (size_t)L * MAX_B, 0, sizeof(u64) * MAX_B, st));
-        const int lev0 = L;
-        L = L + 1;
-        if ((rc = enqueue_levels(lev0, st))) return rc;
+    for (;;) {
+        const SelectResult& h = *c->h_res;
+        if (h.halt) {
+            // re-run the halted level lh the paper's way at level index lh + 2
+            // (its input is level lh's input; index lh + 2 writes the buffer
+            // the halted level wrote, never the one it reads)
+            ++extra_rounds;
+            const int lh = h.halt - 1, lev_new = lh + 2;
+            double m = (double)h.n_level[lh];
+            int L2 = lev_new;
+            while (m > (double)B && L2 < SS_MAX_LEVELS - 2) {
+                m = m * 1.5 / (L2 ? bd : b0);
+                ++L2;
+            }
+            if (L2 >= SS_MAX_LEVELS - 2) return fail(c, SS_ERR_INTERNAL, "recursion too deep after a halt");
+            CK(cudaMemsetAsync(&c->d_res->done, 0, sizeof(int), st));
+            CK(cudaMemsetAsync(&c->d_res->halt, 0, sizeof(int), st));
+            CK(cudaMemcpyAsync(c->d_ctl + lev_new, c->d_ctl + lh + 1, sizeof(LevelCtl), cudaMemcpyDeviceToDevice, st));
+            CK(cudaMemsetAsync(c->d_totals + (size_t)lev_new * MAX_B, 0, sizeof(u64) * MAX_B * (L2 - lev_new + 1), st));
+            std::fill(plan.spec_plan, plan.spec_plan + SS_MAX_LEVELS, false);
+            plan.lev_first = lev_new;
+            plan.sample0 = nullptr;
+            plan.L = L = L2;
+            const T* first_in = lh == 0 ? d : reinterpret_cast<const T*>(c->d_buf[(lh - 1) & 1]);
+            if ((rc = enqueue_exact_levels<T>(c, plan, first_in, lev_new, st))) return rc;
+        } else if (!h.done) {
+            ++extra_rounds;
+            if (!h.incomplete || L >= SS_MAX_LEVELS - 2)
+                return fail(c, SS_ERR_INTERNAL, "recursion did not terminate");
+            CK(cudaMemsetAsync(&c->d_res->incomplete, 0, sizeof(int), st));
+            CK(cudaMemsetAsync(c->d_totals + (size_t)L * MAX_B, 0, sizeof(u64) * MAX_B, st));
+            const int lev0 = L;
+            L = L + 1;
+            if ((rc = enqueue_levels(lev0, st))) return rc;
+        } else {
+            break;
+        }
         if ((rc = enqueue_publish(c, st))) return rc;
         if ((rc = wait_publish(c, st))) return rc;
     }
@@ -813,12 +902,9 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
         const double nl = (double)r.n_level[l], nn = (double)r.n_level[l + 1];
         const bool last_eq = r.eq_exit && l == r.levels - 1;
         if (r.spec_levels >> l & 1) {
-            bytes += Sz * nl;                           // count reads the level once
-            if (!last_eq) {
-                if (r.fused_levels >> l & 1) bytes += Sz * nn;           // window copy written by the count
-                else bytes += 2.0 * Sz * nl;            // miss: the level is copied and re-run
-            }
-            continue;
+            bytes += Sz * nl;                           // the fused pass reads the level once
+            if (!last_eq && (r.fused_levels >> l & 1)) bytes += Sz * nn;   // and writes the window
+            continue;                                   // (a miss halts: the level is re-run from its input)
         }
         bytes += Sz * nl + nl;                          // count: read + oracle write
         if (!last_eq) bytes += nl + 2.0 * Sz * nn;      // oracle read + gather + write

@@ -46,6 +46,7 @@ ss_status run_sharded(ss_context* c, const T* d, u64 n_local, u64 k, void* h_res
     const float z = std::min(c->cfg.spec_z, 16.0f);   // (a window can never cover a whole sample of 4096)
     ss_status rc;
     if ((rc = ensure_small(c))) return rc;
+    if (c->cfg.profile && (rc = prof_init(c))) return rc;
     c->launches = 0;
     c->d2h = 0;
     // workspace: ping-pong level buffers (a level's window plus its chunk
@@ -77,9 +78,32 @@ ss_status run_sharded(ss_context* c, const T* d, u64 n_local, u64 k, void* h_res
         return SS_OK;
     };
 
+    // The plan must be the same on every rank (every rank enqueues the same
+    // collectives), so it is made from a number every rank knows: the size of
+    // the union.  The first call after ss_comm_init exchanges the sizes and
+    // reads N back (one host round trip); later calls plan with the N of the
+    // previous call (published with its result) -- a different N only makes
+    // a level a pass-through or adds one after the hand-off, identically on
+    // every rank.
+    CK(launch_pdl(init_kernel<T>, dim3(1), dim3(256), 0, st, c->d_ctl, (int)(SS_MAX_LEVELS + 1), c->d_totals,
+                  (int)(SS_MAX_LEVELS * MAX_B), c->d_res, n_local, k, 0, d, 0, (u64)c->cfg.seed, (K*)nullptr));
+    CKLAUNCH("init_kernel");
+    CK(launch_pdl(dist_sizes_kernel, dim3(1), dim3(32), 0, st, dd + DistLayout::sizes_send, P, R, n_local));
+    CKLAUNCH("dist_sizes_kernel");
+    if ((rc = exchange(dd + DistLayout::sizes_send, sizes_at(0), (size_t)P, 8, st))) return rc;   // exchange 0
+    CK(launch_pdl(dist_check_kernel, dim3(1), dim3(32), 0, st, (const u64*)sizes_at(0), P, k, c->d_res));
+    CKLAUNCH("dist_check_kernel");
+    c->launches += 3;
+    if (!c->dist_n_plan) {
+        u64 hs[DIST_MAX_RANKS] = {};
+        CK(cudaMemcpyAsync(hs, sizes_at(0), sizeof(u64) * P, cudaMemcpyDeviceToHost, st));
+        CK(cudaStreamSynchronize(st));
+        for (int q = 0; q < P; ++q) c->dist_n_plan += hs[q];
+        c->d2h += (int64_t)(sizeof(u64) * P);
+    }
     // plan: sharded levels until the expected survivors fit the gather buffer
     const double f = dist_window_frac(z, DIST_S);
-    double est = (double)n_local * P;
+    double est = (double)c->dist_n_plan;
     int D = 0;
     while (est > (double)G && D < 8) {
         est = est * f * 1.1 + (double)P * c->sms * 32.0;    // window + chunk padding
@@ -117,7 +141,9 @@ ss_status run_sharded(ss_context* c, const T* d, u64 n_local, u64 k, void* h_res
         w.tail = TAIL_EXACT;
         w.cap_out = c->d_buf[lev & 1];
         w.rec = rsend + (size_t)R * DIST_REC;
+        mark(c, lev, 1, 0, q);
         if ((r2 = launch_window<T>(c, 0, in, w, q))) return r2;
+        mark(c, lev, 1, 1, q);                     // profile 1/2: the level's fused kernel
         if ((r2 = exchange(rsend, rrecv, (size_t)P * DIST_REC, 8, q))) return r2;    // exchange 2
         CK(launch_pdl(dist_decide_kernel<T>, dim3(1), dim3(32), 0, q, ctl, c->d_ctl + lev + 1, c->d_res,
                       (const u64*)rrecv, P, R, sizes_at(lev + 1), lev));
@@ -158,15 +184,6 @@ ss_status run_sharded(ss_context* c, const T* d, u64 n_local, u64 k, void* h_res
 
     int L_tail = tail_levels(est);
     if (D + 1 + L_tail >= SS_MAX_LEVELS - 2) return fail(c, SS_ERR_INTERNAL, "sharded plan too deep");
-    CK(launch_pdl(init_kernel<T>, dim3(1), dim3(256), 0, st, c->d_ctl, (int)(SS_MAX_LEVELS + 1), c->d_totals,
-                  (int)(SS_MAX_LEVELS * MAX_B), c->d_res, n_local, k, 0, d, 0, (u64)c->cfg.seed, (K*)nullptr));
-    CKLAUNCH("init_kernel");
-    CK(launch_pdl(dist_sizes_kernel, dim3(1), dim3(32), 0, st, dd + DistLayout::sizes_send, P, R, n_local));
-    CKLAUNCH("dist_sizes_kernel");
-    if ((rc = exchange(dd + DistLayout::sizes_send, sizes_at(0), (size_t)P, 8, st))) return rc;   // exchange 0
-    CK(launch_pdl(dist_check_kernel, dim3(1), dim3(32), 0, st, (const u64*)sizes_at(0), P, k, c->d_res));
-    CKLAUNCH("dist_check_kernel");
-    c->launches += 3;
     if ((rc = enqueue(0, D, L_tail, st))) return rc;
     if ((rc = enqueue_publish(c, st))) return rc;
     if ((rc = wait_publish(c, st))) return rc;
@@ -196,6 +213,7 @@ ss_status run_sharded(ss_context* c, const T* d, u64 n_local, u64 k, void* h_res
         ++extra;
     }
     const SelectResult& r = *c->h_res;
+    c->dist_n_plan = r.dist_n;                 // the next call's plan (identical on every rank)
     std::memcpy(h_result, &r.bits, sizeof(T));
     ss_stats& S = c->stats;
     std::memset(&S, 0, sizeof(S));
@@ -236,5 +254,6 @@ ss_status run_sharded(ss_context* c, const T* d, u64 n_local, u64 k, void* h_res
     S.d2h_bytes = c->d2h;
     c->launches_total += c->launches;
     c->calls_total += 1;
+    prof_collect(c);
     return SS_OK;
 }

@@ -262,18 +262,20 @@ def test_incomplete_fallback(dtype, cuda_device):
 @pytest.mark.parametrize("dtype", [np.float32, np.float64, np.int32, np.int64])
 def test_fused_window_miss_path(dtype, cuda_device):
     """A level-0 window predicted from a poisoned sample misses rank k: the
-    level is re-run with the paper's tree (ss_stats: spec bit set, hit bit
-    clear) and the answer is still exact."""
+    chain halts and the host re-runs the level with the paper's tree
+    (ss_stats: spec bit set, hit bit clear, one extra round) and the answer
+    is still exact."""
     import paper_conf_ipps_ribizela19_b200 as ss
     c = ss.Context(0)
     try:
         n = (1 << 22) + 1
-        s = 4096
+        s = 16384                                     # the fused level's sample (K1w)
         x = _poisoned(n, dtype, 6, c.config["seed"], s)
         xd = _dev(x)
         for k in (n // 2, n - 1):
             assert _bits(c.select(xd, k)) == _bits(oracle.select(x, k)), k
             st = c.stats()
             assert st["spec_levels"] & 1 and not st["fused_levels"] & 1, st
+            assert st["incomplete_rounds"] >= 1, st
     finally:
         c.close()
