@@ -272,7 +272,7 @@ def test_fused_window_miss_path(dtype, cuda_device):
         s = 16384                                     # the fused level's sample (K1w)
         x = _poisoned(n, dtype, 6, c.config["seed"], s)
         xd = _dev(x)
-        for k in (n // 2, n - 1):
+        for k in (n // 2, n // 3):   # (near n-1 the window [poisoned key, +inf) holds k: a hit)
             assert _bits(c.select(xd, k)) == _bits(oracle.select(x, k)), k
             st = c.stats()
             assert st["spec_levels"] & 1 and not st["fused_levels"] & 1, st
