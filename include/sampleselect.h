@@ -132,6 +132,9 @@ typedef struct {
                                           (n_level[l] for l < shard_levels are global sizes,
                                           n_level[shard_levels] the gathered size) */
     int32_t shard_ranks;               /* ss_select_sharded: ranks of the communicator */
+    int64_t workspace_bytes;           /* ss_select: device bytes the context owns after the call
+                                          (level buffers sized for the planned survivors; they
+                                          grow only when a level would not fit) */
 } ss_stats;
 
 /* ---- context --------------------------------------------------------- */

@@ -53,7 +53,8 @@ class SSStats(ctypes.Structure):
                 ("spec_levels", ctypes.c_int32), ("fused_levels", ctypes.c_int32),
                 ("upper_greater", ctypes.c_int64), ("ms_upper_gather", ctypes.c_float),
                 ("ms_quick", ctypes.c_float), ("incomplete_rounds", ctypes.c_int32),
-                ("shard_levels", ctypes.c_int32), ("shard_ranks", ctypes.c_int32)]
+                ("shard_levels", ctypes.c_int32), ("shard_ranks", ctypes.c_int32),
+                ("workspace_bytes", ctypes.c_int64)]
 
 
 class SSError(RuntimeError):

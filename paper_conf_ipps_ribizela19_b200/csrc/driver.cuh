@@ -234,6 +234,26 @@ ss_status grow(ss_context* c, void** p, size_t* cap, size_t need) {
     return SS_OK;
 }
 
+// Grow *p to `need` bytes keeping its first `keep` bytes (a stream-ordered
+// device copy; the old block is freed once the copy is done).
+ss_status grow_keep(ss_context* c, void** p, size_t* cap, size_t need, size_t keep, cudaStream_t st) {
+    if (*cap >= need && *p) return SS_OK;
+    void* old = *p;
+    *p = nullptr;
+    *cap = 0;
+    ss_status rc = grow(c, p, cap, need);
+    if (rc) return rc;
+    if (old) {
+        if (keep) CK(cudaMemcpyAsync(*p, old, keep, cudaMemcpyDeviceToDevice, st));
+        CK(cudaStreamSynchronize(st));
+        cudaFree(old);
+    }
+    return SS_OK;
+}
+
+// Device bytes the context owns (ss_stats.workspace_bytes).
+size_t workspace_bytes(const ss_context* c);
+
 // count/filter grid: resident CTAs of the count kernel x #SMs (one wave)
 // (the occupancy is cached per context: a context belongs to one device and
 // one host thread, so no cache is shared between threads)
@@ -271,17 +291,17 @@ ss_status launch_count(ss_context* c, int H, const T* in, CountArgs& a, cudaStre
     return SS_OK;
 }
 
-// fused-filter count kernel: one CTA per SM, KW_STASH bytes of stash
+// fused count + filter kernel: one CTA per SM, KW_SMEM bytes (TMA ring + stash)
 template <typename T, bool APX = false>
 ss_status launch_window(ss_context* c, int /*H*/, const T* in, CountArgs a, cudaStream_t st) {
     a.grid = (u32)c->sms * (u32)KW_MINB;
     bool& attr_set = c->kw_attr[dt_code<T>() - 1][APX ? 1 : 0];
     if (!attr_set) {
         CK(cudaFuncSetAttribute(window_kernel<T, APX>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)KW_STASH));
+                                (int)KW_SMEM));
         attr_set = true;
     }
-    CK(launch_pdl(window_kernel<T, APX>, dim3(a.grid), dim3(KW_THREADS), KW_STASH, st, in, a));
+    CK(launch_pdl(window_kernel<T, APX>, dim3(a.grid), dim3(KW_THREADS), KW_SMEM, st, in, a));
     CKLAUNCH("window_kernel");
     return SS_OK;
 }
@@ -581,6 +601,7 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
     typedef typename Traits<T>::Key K;
     ss_status rc;
     const T* in = lev0 > p.lev_first ? reinterpret_cast<const T*>(c->d_buf[(lev0 - 1) & 1]) : first_in;
+    const u64 cap_limit = std::min(c->cap_buf[0], c->cap_buf[1]) / sizeof(T);   // elements per level buffer
     int lev = lev0;
     for (; lev < p.L; ++lev) {
         const int b = lev ? p.bd : p.b0, H = log2i(b);
@@ -610,6 +631,7 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
             w.s_next = sl_next;
             w.seed = (u64)c->cfg.seed;
             w.halt_on_miss = 1;
+            w.cap_limit = cap_limit;
             mark(c, lev, 1, 0, q);
             if ((rc = launch_window<T>(c, H, in, w, q))) return rc;
             mark(c, lev, 1, 1, q);
@@ -634,6 +656,7 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
         a.lut_stats = lev == 0 ? c->d_res->lut_stats : nullptr;
         a.level = lev;
         a.tail = TAIL_EXACT;
+        a.cap_limit = cap_limit;
         if (wide) {
             if ((rc = launch_k1_wide<T>(c, in, lev, sl, p.B, q, pre_this))) return rc;
             if (lev == 0) {
@@ -692,13 +715,26 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     if (c->cfg.profile && (rc = prof_init(c))) return rc;
     c->launches = 0;
     c->d2h = 0;
-    if ((rc = grow(c, (void**)&c->d_oracles, &c->cap_oracles, n + 64))) return rc;
-    // survivor ping-pong buffers: a level's survivors never exceed its input
-    for (int i = 0; i < 2; ++i)
-        if ((rc = grow(c, &c->d_buf[i], &c->cap_buf[i], n * sizeof(T)))) return rc;
     bool spec_plan[SS_MAX_LEVELS] = {};
     const int sf = fused_sample(c->cfg);
     int L = expected_levels(c, n, b0, bd, sf, sf, B, spec_plan);
+    // workspace (reading R16: the paper keeps aux storage <= n/4 elements):
+    // the two level buffers hold the planned level-1 survivors with 2x slack
+    // (a level whose survivors would not fit halts before writing past them;
+    // the host grows the buffers to n and re-runs it), the oracle bytes the
+    // largest planned paper level
+    {
+        const double f0 = window_frac(spec_params(c).z, sf);
+        const double est1 = L == 0 ? 0.0 : spec_plan[0] ? (double)n * 1.2 * f0 + (double)c->sms * 4096.0
+                                                         : (double)n * 1.5 / b0;
+        const u64 cap_el = std::min<u64>(n, std::max<u64>((u64)(2.0 * est1), (u64)1 << 20));
+        for (int i = 0; i < 2; ++i)
+            if ((rc = grow(c, &c->d_buf[i], &c->cap_buf[i], cap_el * sizeof(T)))) return rc;
+        bool paper_deep = false;
+        for (int l = 1; l < L; ++l) paper_deep |= !spec_plan[l];
+        const u64 orc = L > 0 && !spec_plan[0] ? n : paper_deep ? cap_el : 0;
+        if ((rc = grow(c, (void**)&c->d_oracles, &c->cap_oracles, orc + 64))) return rc;
+    }
     // level 0's sample is gathered by the init kernel (spread over the grid)
     // when K1w or the wide K1 takes it from memory
     const int s_init = L > 0 && spec_plan[0] ? sf : s;
@@ -847,8 +883,16 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             // (its input is level lh's input; index lh + 2 writes the buffer
             // the halted level wrote, never the one it reads)
             ++extra_rounds;
-            const int lh = h.halt - 1, lev_new = lh + 2;
-            double m = (double)h.n_level[lh];
+            const int lh = (h.halt & 0xFFFF) - 1, lev_new = lh + 2;
+            const u64 nh = (u64)h.n_level[lh];
+            if (h.halt & SS_HALT_OVERFLOW) {        // grow the level buffers to n, keeping level lh's input
+                const size_t keep = lh ? (size_t)nh * sizeof(T) : 0;
+                const int bi = (lh - 1) & 1;
+                if ((rc = grow_keep(c, &c->d_buf[bi], &c->cap_buf[bi], n * sizeof(T), lh ? keep : 0, st))) return rc;
+                if ((rc = grow_keep(c, &c->d_buf[bi ^ 1], &c->cap_buf[bi ^ 1], n * sizeof(T), 0, st))) return rc;
+            }
+            if ((rc = grow(c, (void**)&c->d_oracles, &c->cap_oracles, nh + 64))) return rc;
+            double m = (double)nh;
             int L2 = lev_new;
             while (m > (double)B && L2 < SS_MAX_LEVELS - 2) {
                 m = m * 1.5 / (L2 ? bd : b0);
@@ -891,6 +935,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     S.spec_levels = (int32_t)r.spec_levels;
     S.fused_levels = (int32_t)r.fused_levels;
     S.incomplete_rounds = extra_rounds;
+    S.workspace_bytes = (int64_t)workspace_bytes(c);
     if (r.spec_err) return fail(c, SS_ERR_INTERNAL, "fused filter: captured count != window total");
     double bytes = 0;
     const double Sz = (double)sizeof(T);
@@ -1317,6 +1362,17 @@ ss_status run_quick(ss_context* c, const T* d, u64 n, u64 k, void* h_result, int
 }
 
 
+
+size_t workspace_bytes(const ss_context* c) {
+    size_t b = c->cap_oracles + c->cap_buf[0] + c->cap_buf[1] + c->cap_stage + c->cap_multi + 2 * c->cap_qsbuf +
+               c->cap_gather[0] + c->cap_gather[1] + c->cap_dist;
+    if (c->d_ctl)   // the fixed per-context arrays (ensure_small)
+        b += sizeof(LevelCtl) * (SS_MAX_LEVELS + 1) + sizeof(SelectResult) + sizeof(u64) * SS_MAX_LEVELS * MAX_B +
+             sizeof(u32) * (size_t)MAX_GRID * MAX_B + 2 * sizeof(u64) * SS_MAX_LEVELS * MAX_B +
+             (size_t)SS_MAX_LEVELS * MAX_B + sizeof(u64) * SS_MAX_LEVELS * MAX_S + sizeof(u64) * MAX_S +
+             sizeof(u64) * SS_MAX_LEVELS * MAX_S + K2_IMAGE_SLOT * SS_MAX_LEVELS;
+    return b;
+}
 
 #include "sharded.cuh"
 

@@ -80,15 +80,15 @@ qs_pivot_kernel(const T* __restrict__ in0, const T* __restrict__ buf_in, QsCtl* 
                 int level) {
     typedef typename Traits<T>::Key K;
     __shared__ __align__(16) K keys[QS_SAMPLE];
-    __shared__ u32 hist[32 * 256];
+    __shared__ __align__(16) u32 hist[32 * 256];
     __shared__ u32 misc[16];
-    __shared__ K red[64];
+    __shared__ K red[66];
     __shared__ u32 misc_rank[QS_SAMPLE];
     if (c->done) return;
     const u64 n = c->n;
     const T* in = qs_input(in0, buf_in, c, level);
     if (n <= B) {                                 // Fig. 1 lines 2-5: base case
-        K r = block_radix_select<T>(in, (u32)n, (u32)c->k, hist, misc, red);
+        K r = block_select_base<T>(in, (u32)n, (u32)c->k, hist, misc, red);
         if (threadIdx.x == 0) {
             c->n_level[level] = n;
             c->n_out[level] = 0;
