@@ -457,10 +457,13 @@ SpecCfg spec_params(const ss_context* c) {
 }
 
 // Fused-level sample sizes (K1w): the configured sample_size if set (at least
-// 1024), else 16384 -- the window is ~6 z / sqrt(s) of the level.
-inline int fused_sample(const ss_config& cfg) {
+// 1024), else 16384 at level 0 and 4096 deeper -- the window is ~6 z / sqrt(s)
+// of the level, and K1w's cost (one CTA) grows with s: level 0's window
+// decides the largest write and the next level's size, deeper levels are
+// small enough that a cheaper K1w wins.
+inline int fused_sample(const ss_config& cfg, int level) {
     if (cfg.sample_size > 0) return std::max(1024, std::min(cfg.sample_size, 16384));
-    return 16384;
+    return level ? 4096 : 16384;
 }
 
 inline double window_frac(float z, int s) {
@@ -716,8 +719,8 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     c->launches = 0;
     c->d2h = 0;
     bool spec_plan[SS_MAX_LEVELS] = {};
-    const int sf = fused_sample(c->cfg);
-    int L = expected_levels(c, n, b0, bd, sf, sf, B, spec_plan);
+    const int sf = fused_sample(c->cfg, 0), sfd = fused_sample(c->cfg, 1);
+    int L = expected_levels(c, n, b0, bd, sf, sfd, B, spec_plan);
     // workspace (reading R16: the paper keeps aux storage <= n/4 elements):
     // the two level buffers hold the planned level-1 survivors with 2x slack
     // (a level whose survivors would not fit halts before writing past them;
@@ -753,7 +756,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     };
     ExactPlan plan{};
     plan.b0 = b0; plan.bd = bd; plan.s = s; plan.s_deep = s_deep; plan.B = B; plan.L = L;
-    plan.sf0 = sf; plan.sfd = sf;
+    plan.sf0 = sf; plan.sfd = sfd;
     std::copy(spec_plan, spec_plan + SS_MAX_LEVELS, plan.spec_plan);
     plan.sample0 = sample0;
     plan.lev_first = 0;

@@ -177,7 +177,9 @@ def test_step_count_misaligned_view(ctx):
         ctx.step_filter(xd, orc, j, out, cnt)
         m = int(cnt.item())
         assert m == counts_o[j]
-        assert np.array_equal(out[:m].cpu().numpy(), oracle.filter_bucket(ref, orc_o, j))
+        # the filter is not stable (R15, like the paper's shared counter): compare the multisets
+        assert np.array_equal(np.sort(out[:m].cpu().numpy().view(np.uint32)),
+                              np.sort(oracle.filter_bucket(ref, orc_o, j).view(np.uint32)))
 
 
 # ------------------------------------------------ configurations / paths --
