@@ -457,10 +457,11 @@ SpecCfg spec_params(const ss_context* c) {
 }
 
 // Fused-level sample sizes (K1w): the configured sample_size if set (at least
-// 1024), else 16384 at level 0 and 4096 deeper -- the window is ~6 z / sqrt(s)
-// of the level, and K1w's cost (one CTA) grows with s: level 0's window
-// decides the largest write and the next level's size, deeper levels are
-// small enough that a cheaper K1w wins.
+// 1024), else 16384 at level 0 -- the window is ~6 z / sqrt(s) of the level,
+// and level 0's window decides the largest write and the next level's size --
+// and, deeper, the smallest of 4096 / 8192 / 16384 whose expected window fits
+// the base case (saving a whole level), else 4096: K1w runs on one CTA and
+// its cost grows with s.
 inline int fused_sample(const ss_config& cfg, int level) {
     if (cfg.sample_size > 0) return std::max(1024, std::min(cfg.sample_size, 16384));
     return level ? 4096 : 16384;
@@ -474,18 +475,28 @@ inline double window_frac(float z, int s) {
 // input (the bucket holding k is size-biased, ~1.1 for s / b = 16; 1.5 is
 // slack); a fused level keeps its window (<= window_frac of it, plus chunk
 // padding).  Levels with at least spec_min_n elements (host estimate) are
-// fused when fused_filter is on.  An under-estimate is caught on the device
-// (the final K1 flags "incomplete") and more levels are enqueued.
-int expected_levels(const ss_context* c, u64 n, int b0, int bd, int sf0, int sfd, u32 B, bool* spec_plan) {
+// fused when fused_filter is on; sf_plan[l] is a fused level's sample size.
+// An under-estimate is caught on the device (the final K1 flags
+// "incomplete") and more levels are enqueued.
+int expected_levels(const ss_context* c, u64 n, int b0, int bd, u32 B, bool* spec_plan, int* sf_plan) {
     const SpecCfg sp = spec_params(c);
+    const double pad = (double)c->sms * 32.0;
     int L = 0;
     double m = (double)n;
     while (m > (double)B && L < SS_MAX_LEVELS - 2) {
         const int b = L ? bd : b0;
-        const double f = window_frac(sp.z, L ? sfd : sf0);
+        int sf = fused_sample(c->cfg, L);
+        if (L && c->cfg.sample_size <= 0)
+            for (int cand = 4096; cand <= 16384; cand *= 2)
+                if (m * 1.2 * window_frac(sp.z, cand) + pad <= 0.9 * B) {
+                    sf = cand;
+                    break;
+                }
+        const double f = window_frac(sp.z, sf);
         const bool spec = sp.min_n != ~0ull && m >= (double)sp.min_n && f <= sp.max_frac;
         if (spec_plan) spec_plan[L] = spec;
-        m = spec ? m * 1.2 * f + (double)c->sms * 32.0 : m * 1.5 / b;
+        if (sf_plan) sf_plan[L] = sf;
+        m = spec ? m * 1.2 * f + pad : m * 1.5 / b;
         ++L;
     }
     return L;
@@ -564,7 +575,7 @@ ss_status launch_image(ss_context* c, int H, int lev, int s, int fixup, cudaStre
 // level l > p.lev_first reads the buffer level l-1 wrote (d_buf[(l-1) & 1]).
 struct ExactPlan {
     int b0, bd, s, s_deep;
-    int sf0, sfd;                     // sample sizes of fused levels: level 0, deeper levels
+    int sfs[SS_MAX_LEVELS];           // sample size of each fused level
     u32 B;
     int L;                            // levels [.., L) are enqueued, then the final K1
     bool spec_plan[SS_MAX_LEVELS];    // level l is a fused level
@@ -573,7 +584,7 @@ struct ExactPlan {
 };
 
 inline int plan_sample(const ExactPlan& p, int lev) {
-    if (p.spec_plan[lev]) return lev ? p.sfd : p.sf0;
+    if (p.spec_plan[lev]) return p.sfs[lev];
     return lev ? p.s_deep : p.s;
 }
 
@@ -719,8 +730,9 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     c->launches = 0;
     c->d2h = 0;
     bool spec_plan[SS_MAX_LEVELS] = {};
-    const int sf = fused_sample(c->cfg, 0), sfd = fused_sample(c->cfg, 1);
-    int L = expected_levels(c, n, b0, bd, sf, sfd, B, spec_plan);
+    int sf_plan[SS_MAX_LEVELS] = {};
+    int L = expected_levels(c, n, b0, bd, B, spec_plan, sf_plan);
+    const int sf = sf_plan[0] ? sf_plan[0] : fused_sample(c->cfg, 0);
     // workspace (reading R16: the paper keeps aux storage <= n/4 elements):
     // the two level buffers hold the planned level-1 survivors with 2x slack
     // (a level whose survivors would not fit halts before writing past them;
@@ -756,7 +768,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     };
     ExactPlan plan{};
     plan.b0 = b0; plan.bd = bd; plan.s = s; plan.s_deep = s_deep; plan.B = B; plan.L = L;
-    plan.sf0 = sf; plan.sfd = sfd;
+    std::copy(sf_plan, sf_plan + SS_MAX_LEVELS, plan.sfs);
     std::copy(spec_plan, spec_plan + SS_MAX_LEVELS, plan.spec_plan);
     plan.sample0 = sample0;
     plan.lev_first = 0;
@@ -857,9 +869,12 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             // patch them into the cached graph
             u64 kk = k;
             const T* dd = d;
-            std::memcpy(ge->init_store + ge->k_offset, &kk, sizeof(u64));
-            std::memcpy(ge->init_store + ge->d_offset, &dd, sizeof(const T*));
-            CK(cudaGraphExecKernelNodeSetParams(ge->exec, ge->init_node, &ge->init_params));
+            if (std::memcmp(ge->init_store + ge->k_offset, &kk, sizeof(u64)) ||
+                std::memcmp(ge->init_store + ge->d_offset, &dd, sizeof(const T*))) {   // (unchanged: no update)
+                std::memcpy(ge->init_store + ge->k_offset, &kk, sizeof(u64));
+                std::memcpy(ge->init_store + ge->d_offset, &dd, sizeof(const T*));
+                CK(cudaGraphExecKernelNodeSetParams(ge->exec, ge->init_node, &ge->init_params));
+            }
         }
         ge->stamp = ++c->graph_clock;
         if (c->host_timing) c->ht[0] += now_us() - t_in;
