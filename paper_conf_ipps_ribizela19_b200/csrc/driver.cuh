@@ -486,9 +486,11 @@ int expected_levels(const ss_context* c, u64 n, int b0, int bd, u32 B, bool* spe
     while (m > (double)B && L < SS_MAX_LEVELS - 2) {
         const int b = L ? bd : b0;
         int sf = fused_sample(c->cfg, L);
+        // (the window's share of the level varies by ~5 % at s = 16384; a
+        // CTA pads half a 32-element chunk on average)
         if (L && c->cfg.sample_size <= 0)
             for (int cand = 4096; cand <= 16384; cand *= 2)
-                if (m * 1.2 * window_frac(sp.z, cand) + pad <= 0.9 * B) {
+                if (m * 1.1 * window_frac(sp.z, cand) + pad / 2 <= (double)B) {
                     sf = cand;
                     break;
                 }
