@@ -323,9 +323,9 @@ u32 grid_for(ss_context* c, int H) {
 
 // K1's dynamic smem holds the s sample keys (the base case keeps its keys in registers)
 template <typename T>
-size_t k1_smem(int s, u32 /*B*/) {
+size_t k1_smem(int s, u32 B) {            // the sample, or the base case's B keys
     typedef typename Traits<T>::Key K;
-    return (size_t)s * sizeof(K);
+    return (size_t)std::max<u32>((u32)s, B) * sizeof(K);
 }
 
 template <typename T>
@@ -340,6 +340,13 @@ ss_status set_k1_attrs(ss_context* c) {
                             (int)(K1C_CHUNK * sizeof(K))));
     CK(cudaFuncSetAttribute(sample_merge_rank_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                             (int)(16384 * sizeof(K))));
+    CK(cudaFuncSetAttribute(qs_pivot_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)(16384 * sizeof(K))));
+    CK(cudaFuncSetAttribute(window_select_kernel<T, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(16384 * sizeof(K))));
+    CK(cudaFuncSetAttribute(window_select_kernel<T, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(16384 * sizeof(K))));
+    CK(cudaFuncSetAttribute(window_select_kernel<T, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(16384 * sizeof(K))));
+    CK(cudaFuncSetAttribute(window_select_kernel<T, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(16384 * sizeof(K))));
+    CK(cudaFuncSetAttribute(window_select_kernel<T, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(16384 * sizeof(K))));
     return SS_OK;
 }
 
@@ -597,7 +604,8 @@ ss_status launch_wsel(ss_context* c, const T* in, int lev, int s, u32 B, const v
     mark(c, lev, 0, 0, q);
 #define SS_WSEL_CASE(E)                                                                                    \
     case E:                                                                                                \
-        CK(launch_pdl(window_select_kernel<T, E>, dim3(1), dim3(WS_THREADS), 0, q, in, c->d_ctl + lev,     \
+        CK(launch_pdl(window_select_kernel<T, E>, dim3(1), dim3(WS_THREADS), k1_smem<T>(s, B), q, in,      \
+                      c->d_ctl + lev,                                                                      \
                       c->d_ctl + lev + 1, c->d_res, reinterpret_cast<const K*>(pre), B, (u64)c->cfg.seed, \
                       lev, sp.z, sp.max_frac));                                                            \
         break;
@@ -631,7 +639,9 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
                                       ? (const void*)(reinterpret_cast<K*>(c->d_presample) + (size_t)lev * MAX_S)
                                       : nullptr);
         if (p.spec_plan[lev]) {               // fused level: K1w + count/filter in one pass
-            if ((rc = launch_wsel<T>(c, in, lev, sl, p.B, pre_this, q))) return rc;
+            const void* pre_buf = pre_this ? pre_this
+                                           : (const void*)(reinterpret_cast<K*>(c->d_presample) + (size_t)lev * MAX_S);
+            if ((rc = launch_wsel<T>(c, in, lev, sl, p.B, pre_buf, q))) return rc;
             const SpecCfg sp = spec_params(c);
             CountArgs w{};
             w.ctl = c->d_ctl + lev;
@@ -1339,7 +1349,8 @@ ss_status run_quick(ss_context* c, const T* d, u64 n, u64 k, void* h_result, int
     for (;; batch = QS_BATCH) {
         for (int q = 0; q < batch; ++q, ++level) {
             const T* bin = buf[(level + 1) & 1];      // level l reads buffer (l-1)&1 (level 0: d)
-            qs_pivot_kernel<T><<<1, 1024, 0, st>>>(d, bin, c->d_qs, B, c->cfg.seed, level);
+            qs_pivot_kernel<T><<<1, 1024, (size_t)B * sizeof(typename Traits<T>::Key), st>>>(d, bin, c->d_qs, B,
+                                                                                          c->cfg.seed, level);
             qs_partition_kernel<T, IPT><<<grid, QP_THREADS, 0, st>>>(d, bin, buf[level & 1], c->d_qs, level);
             qs_decide_kernel<T><<<1, 1, 0, st>>>(c->d_qs, level);
             CK(cudaGetLastError());

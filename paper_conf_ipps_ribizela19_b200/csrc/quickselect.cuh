@@ -84,11 +84,12 @@ qs_pivot_kernel(const T* __restrict__ in0, const T* __restrict__ buf_in, QsCtl* 
     __shared__ u32 misc[16];
     __shared__ K red[66];
     __shared__ u32 misc_rank[QS_SAMPLE];
+    extern __shared__ __align__(16) unsigned char qs_smem[];   // the base case's keys (B of them)
     if (c->done) return;
     const u64 n = c->n;
     const T* in = qs_input(in0, buf_in, c, level);
     if (n <= B) {                                 // Fig. 1 lines 2-5: base case
-        K r = block_select_base<T>(in, (u32)n, (u32)c->k, hist, misc, red);
+        K r = block_select_base<T>(in, (u32)n, (u32)c->k, reinterpret_cast<K*>(qs_smem), hist, misc, red);
         if (threadIdx.x == 0) {
             c->n_level[level] = n;
             c->n_out[level] = 0;

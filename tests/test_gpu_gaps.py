@@ -281,3 +281,50 @@ def test_fused_window_miss_path(dtype, cuda_device):
             assert st["incomplete_rounds"] >= 1, st
     finally:
         c.close()
+
+
+# ------------------------------------------------------ workspace (R16) --
+def test_workspace_is_sized_for_the_survivors(cuda_device):
+    """Round 1 kept two n-element survivor buffers and n oracle bytes; the
+    level buffers are now sized for the planned level-1 survivors."""
+    import paper_conf_ipps_ribizela19_b200 as ss
+    c = ss.Context(0)
+    try:
+        n = 1 << 24
+        x = datagen.uniform(n, np.float32, seed=3)
+        xd = _dev(x)
+        for k in (n // 2, 5, n - 3):
+            assert _bits(c.select(xd, k)) == _bits(oracle.select(x, k))
+        st = c.stats()
+        assert st["workspace_bytes"] <= 0.5 * n * 4 + (32 << 20), st["workspace_bytes"]
+    finally:
+        c.close()
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.int64])
+def test_level_overflow_grows_and_reruns(dtype, cuda_device):
+    """40 % of the input is one value just above rank k's neighbourhood: the
+    fused window [v, v') holds the whole run, far more than the buffers sized
+    for a ~3 % window -- the level halts before writing past them, the host
+    grows the buffers and re-runs it; the answer stays exact."""
+    import paper_conf_ipps_ribizela19_b200 as ss
+    c = ss.Context(0)
+    try:
+        n = 1 << 24
+        rng = np.random.default_rng(11)
+        if np.dtype(dtype).kind == "f":
+            x = datagen.uniform(n, dtype, seed=12)
+            v = dtype(0.5)
+        else:
+            x = datagen.int_uniform(n, dtype, seed=12)
+            v = dtype(0)
+        x[rng.random(n) < 0.4] = v
+        xd = _dev(x)
+        below = int(np.sum(x < v))
+        k = below + int(0.4 * n) - 1000            # inside the run, near its top: the window reaches past it
+        ref = _bits(oracle.select(x, k))
+        assert _bits(c.select(xd, k)) == ref
+        for kk in (below - 5, below + int(0.4 * n) + 50, n // 2):
+            assert _bits(c.select(xd, kk)) == _bits(oracle.select(x, kk)), kk
+    finally:
+        c.close()
