@@ -31,13 +31,28 @@ _NP_DT = {np.dtype(np.float32): _abi.SS_FLOAT32, np.dtype(np.float64): _abi.SS_F
 _NP_OF = {v: k for k, v in _NP_DT.items()}
 
 
+_TORCH_DT = None
+
+
 def _torch_dt(t):
-    import torch
-    m = {torch.float32: _abi.SS_FLOAT32, torch.float64: _abi.SS_FLOAT64,
-         torch.int32: _abi.SS_INT32, torch.int64: _abi.SS_INT64}
-    if t.dtype not in m:
+    global _TORCH_DT
+    if _TORCH_DT is None:
+        import torch
+        _TORCH_DT = {torch.float32: _abi.SS_FLOAT32, torch.float64: _abi.SS_FLOAT64,
+                     torch.int32: _abi.SS_INT32, torch.int64: _abi.SS_INT64}
+    code = _TORCH_DT.get(t.dtype)
+    if code is None:
         raise TypeError(f"unsupported dtype {t.dtype}; use float32/float64/int32/int64")
-    return m[t.dtype]
+    return code
+
+
+def _current_stream(device: int) -> int:
+    """The raw cudaStream_t torch considers current on `device`."""
+    import torch
+    raw = getattr(torch._C, "_cuda_getCurrentRawStream", None)
+    if raw is not None:
+        return raw(device)
+    return torch.cuda.current_stream(device).cuda_stream
 
 
 def _is_tensor(x) -> bool:
@@ -58,6 +73,7 @@ class Context:
         if rc:
             raise SSError(rc, f"ss_create(device={device}) failed (is a CUDA device visible?)")
         self.device = int(device)
+        self._out = {code: np.empty(1, dtype=npdt) for npdt, code in _NP_DT.items()}
         if config:
             self.configure(**config)
 
@@ -79,9 +95,8 @@ class Context:
 
     def _stream(self, stream):
         if stream is not None:
-            return ctypes.c_void_p(stream if isinstance(stream, int) else stream.cuda_stream)
-        import torch
-        return ctypes.c_void_p(torch.cuda.current_stream(self.device).cuda_stream)
+            return stream if isinstance(stream, int) else stream.cuda_stream
+        return _current_stream(self.device)
 
     @property
     def config(self) -> dict:
@@ -138,7 +153,7 @@ class Context:
             if x.device.index != self.device:
                 raise ValueError(f"tensor on cuda:{x.device.index}, context on cuda:{self.device}")
             dt = _torch_dt(x)
-            return dt, ctypes.c_void_p(x.data_ptr()), x.numel(), _NP_OF[dt], True
+            return dt, x.data_ptr(), x.numel(), _NP_OF[dt], True
         a = np.asarray(x)
         if a.ndim != 1 or not a.flags.c_contiguous:
             raise ValueError("input must be a 1-D contiguous array")
@@ -150,9 +165,11 @@ class Context:
     def select(self, x, k: int, stream=None):
         """Element of rank k (0-based; ties take the smallest rank, §II)."""
         dt, p, n, npdt, dev = self._args(x)
-        out = np.empty(1, dtype=npdt)
+        out = self._out[dt]                     # (a per-context result slot: the call is synchronous)
         fn = self._lib.ss_select if dev else self._lib.ss_select_host
-        self._check(fn(self._h, dt, p, n, int(k), ctypes.c_void_p(out.ctypes.data), self._stream(stream)))
+        rc = fn(self._h, dt, p, n, int(k), out.ctypes.data, self._stream(stream))
+        if rc:
+            self._check(rc)
         return out[0]
 
     def approx_select(self, x, k: int, b: int = 1024, stream=None):

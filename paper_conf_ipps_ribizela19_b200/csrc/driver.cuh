@@ -342,11 +342,8 @@ ss_status set_k1_attrs(ss_context* c) {
                             (int)(16384 * sizeof(K))));
     CK(cudaFuncSetAttribute(qs_pivot_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                             (int)(16384 * sizeof(K))));
-    CK(cudaFuncSetAttribute(window_select_kernel<T, 1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(16384 * sizeof(K))));
-    CK(cudaFuncSetAttribute(window_select_kernel<T, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(16384 * sizeof(K))));
-    CK(cudaFuncSetAttribute(window_select_kernel<T, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(16384 * sizeof(K))));
-    CK(cudaFuncSetAttribute(window_select_kernel<T, 8>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(16384 * sizeof(K))));
-    CK(cudaFuncSetAttribute(window_select_kernel<T, 16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(16384 * sizeof(K))));
+    CK(cudaFuncSetAttribute(wsel_cluster_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                            (int)(WC_KEYS * sizeof(K))));
     return SS_OK;
 }
 
@@ -574,7 +571,7 @@ ss_status launch_image(ss_context* c, int H, int lev, int s, int fixup, cudaStre
 // The exact chain of Fig. 1 (L95-127) from level lev0 to the plan's L.  A
 // paper level is K1 (sample + sort, or the base case), the tree image, K2
 // (count + K3/K4 tail) and K5 (filter); a fused level (spec_plan) is K1w (the
-// window straight from the sample, window_select_kernel) and the fused
+// window straight from the sample, wsel_cluster_kernel) and the fused
 // count + filter pass (window_kernel) -- nothing else is enqueued behind it:
 // a miss halts the chain (SelectResult::halt) and the host re-runs that level
 // the paper's way.  Every kernel reads its sizes from the device-resident
@@ -598,23 +595,15 @@ inline int plan_sample(const ExactPlan& p, int lev) {
 }
 
 template <typename T>
-ss_status launch_wsel(ss_context* c, const T* in, int lev, int s, u32 B, const void* pre, cudaStream_t q) {
+ss_status launch_wsel(ss_context* c, const T* in, int lev, int s, u32 B, const void* pre, int final_level,
+                      cudaStream_t q) {
     typedef typename Traits<T>::Key K;
     const SpecCfg sp = spec_params(c);
     mark(c, lev, 0, 0, q);
-#define SS_WSEL_CASE(E)                                                                                    \
-    case E:                                                                                                \
-        CK(launch_pdl(window_select_kernel<T, E>, dim3(1), dim3(WS_THREADS), k1_smem<T>(s, B), q, in,      \
-                      c->d_ctl + lev,                                                                      \
-                      c->d_ctl + lev + 1, c->d_res, reinterpret_cast<const K*>(pre), B, (u64)c->cfg.seed, \
-                      lev, sp.z, sp.max_frac));                                                            \
-        break;
-    switch (s / WS_THREADS) {
-        SS_WSEL_CASE(1) SS_WSEL_CASE(2) SS_WSEL_CASE(4) SS_WSEL_CASE(8) SS_WSEL_CASE(16)
-    default: return fail(c, SS_ERR_INTERNAL, "fused-level sample size must be 1024 * 2^i <= 16384");
-    }
-#undef SS_WSEL_CASE
-    CKLAUNCH("window_select_kernel");
+    CK(launch_pdl(wsel_cluster_kernel<T>, dim3(WC_CTAS), dim3(WS_THREADS), WC_KEYS * sizeof(K), q, in,
+                  c->d_ctl + lev, c->d_ctl + lev + 1, c->d_res, reinterpret_cast<const K*>(pre), (u32)s, B,
+                  (u64)c->cfg.seed, lev, sp.z, sp.max_frac, final_level));
+    CKLAUNCH("wsel_cluster_kernel");
     mark(c, lev, 0, 1, q);
     ++c->launches;
     return SS_OK;
@@ -641,7 +630,7 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
         if (p.spec_plan[lev]) {               // fused level: K1w + count/filter in one pass
             const void* pre_buf = pre_this ? pre_this
                                            : (const void*)(reinterpret_cast<K*>(c->d_presample) + (size_t)lev * MAX_S);
-            if ((rc = launch_wsel<T>(c, in, lev, sl, p.B, pre_buf, q))) return rc;
+            if ((rc = launch_wsel<T>(c, in, lev, sl, p.B, pre_buf, 0, q))) return rc;
             const SpecCfg sp = spec_params(c);
             CountArgs w{};
             w.ctl = c->d_ctl + lev;
@@ -721,7 +710,8 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
         ++c->launches;
         in = out;
     }
-    return launch_k1<T>(c, in, lev, lev ? p.s_deep : p.s, lev ? p.bd : p.b0, 1, p.B, 1, q);
+    // the final level: the base case on one cluster (or the "incomplete" flag)
+    return launch_wsel<T>(c, in, lev, 0, p.B, nullptr, 1, q);
 }
 
 template <typename T>
