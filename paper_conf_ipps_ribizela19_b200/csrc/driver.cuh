@@ -600,7 +600,7 @@ ss_status launch_wsel(ss_context* c, const T* in, int lev, int s, u32 B, const v
     typedef typename Traits<T>::Key K;
     const SpecCfg sp = spec_params(c);
     mark(c, lev, 0, 0, q);
-    CK(launch_pdl(wsel_cluster_kernel<T>, dim3(WC_CTAS), dim3(WS_THREADS), WC_KEYS * sizeof(K), q, in,
+    CK(launch_pdl(wsel_cluster_kernel<T>, dim3(WC_CTAS), dim3(WC_THREADS), WC_KEYS * sizeof(K), q, in,
                   c->d_ctl + lev, c->d_ctl + lev + 1, c->d_res, reinterpret_cast<const K*>(pre), (u32)s, B,
                   (u64)c->cfg.seed, lev, sp.z, sp.max_frac, final_level));
     CKLAUNCH("wsel_cluster_kernel");
