@@ -30,6 +30,10 @@ for _ in range(R):
     acc = tl if acc is None else acc + tl
 tl = acc / R
 names = ["K1", "K2", "K5"]
+if os.environ.get("WS_DEBUG"):
+    import ctypes
+    raw = np.array(ctx.raw_tl(), dtype=np.float64)   # us after init, last call only
+    print("  K1w phases (us after init, last call):", [round(raw[(80 + i) // 3][(80 + i) % 3][1], 2) for i in range(6)])
 if os.environ.get("TL_DEBUG"):
     for sl, nm in ((93, "L1K2 cta start"), (90, "L1K2 prologue end"), (91, "L1K2 main end"), (92, "L1K2 ticket")):
         l, q = divmod(sl, 3)
