@@ -37,7 +37,7 @@
 extern "C" {
 #endif
 
-#define SS_ABI_VERSION 5
+#define SS_ABI_VERSION 6
 #define SS_MAX_LEVELS 32
 
 typedef enum { SS_FLOAT32 = 0, SS_FLOAT64 = 1, SS_INT32 = 2, SS_INT64 = 3 } ss_dtype;
@@ -92,6 +92,10 @@ typedef struct {
     int32_t shard_gather_log2; /* ss_select_sharded: survivors are gathered onto every rank once
                              the level holds at most 2^shard_gather_log2 elements (then the
                              single-GPU levels finish); 0 = default 20, else in [12, 28] */
+    int32_t directed;     /* fused levels after the first: 1 = (default) the previous fused level
+                             counts the keys it copies in 1024 equal key bins and the bin
+                             holding the rank is this level's window (reading R28: exact, no
+                             sample, cannot miss); 0 = every fused level draws a sample. */
 } ss_config;
 
 /* Per-call statistics of the last ss_select / ss_approx_select. */

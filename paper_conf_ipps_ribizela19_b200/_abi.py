@@ -37,7 +37,7 @@ class SSConfig(ctypes.Structure):
                 ("classify", ctypes.c_int32), ("seed", ctypes.c_uint64),
                 ("fused_filter", ctypes.c_int32), ("spec_z", ctypes.c_float),
                 ("spec_min_n", ctypes.c_int64), ("spec_max_frac", ctypes.c_float),
-                ("shard_gather_log2", ctypes.c_int32)]
+                ("shard_gather_log2", ctypes.c_int32), ("directed", ctypes.c_int32)]
 
 
 class SSStats(ctypes.Structure):

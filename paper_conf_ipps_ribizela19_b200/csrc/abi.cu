@@ -79,6 +79,7 @@ ss_status ss_create(int device, ss_context** out) {
     c->cfg.spec_min_n = (int64_t)1 << 16;
     c->cfg.spec_max_frac = 0.25f;
     c->cfg.shard_gather_log2 = 0;
+    c->cfg.directed = 1;
     DevGuard g(device);
     if (cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess) {
         (void)cudaGetLastError();
@@ -187,10 +188,13 @@ ss_status ss_set_config(ss_context* c, const ss_config* cfg) {
         return fail(c, SS_ERR_INVALID_ARGUMENT, "spec_max_frac must be in (0, 1]");
     if (cfg->shard_gather_log2 != 0 && (cfg->shard_gather_log2 < 12 || cfg->shard_gather_log2 > 28))
         return fail(c, SS_ERR_INVALID_ARGUMENT, "shard_gather_log2 must be 0 or in [12, 28]");
+    if (cfg->directed != 0 && cfg->directed != 1)
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "directed must be 0 or 1");
     // captured graphs bake in grid sizes and the fused-filter parameters
     const bool regrid = cfg->ctas_per_sm != c->cfg.ctas_per_sm || cfg->classify != c->cfg.classify ||
                         cfg->fused_filter != c->cfg.fused_filter || cfg->spec_z != c->cfg.spec_z ||
-                        cfg->spec_min_n != c->cfg.spec_min_n || cfg->spec_max_frac != c->cfg.spec_max_frac;
+                        cfg->spec_min_n != c->cfg.spec_min_n || cfg->spec_max_frac != c->cfg.spec_max_frac ||
+                        cfg->directed != c->cfg.directed;
     c->cfg = *cfg;
     if (regrid)                   // captured grid sizes are stale (the other knobs are part of the graph key)
         for (auto& e : c->graphs) {

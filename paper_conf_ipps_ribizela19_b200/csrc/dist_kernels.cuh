@@ -139,7 +139,7 @@ __global__ void dist_decide_kernel(LevelCtl* __restrict__ ctl, LevelCtl* __restr
         res->fused_levels |= 1u << level;
         ctl_next->n = rows[rank * DIST_REC + 2];
         ctl_next->gn = C;
-        ctl_next->k = k - below;
+        ctl_next->k = k - below + (pad_low(klo, kspan) ? C - W : 0ull);   // (padding below the window)
         for (int q = 0; q < P; ++q) sizes_next[q] = rows[q * DIST_REC + 2];
         return;
     }

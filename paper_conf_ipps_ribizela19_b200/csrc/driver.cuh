@@ -478,20 +478,24 @@ inline double window_frac(float z, int s) {
 // The planned levels of an exact call.  A paper level keeps ~1.5 / b of its
 // input (the bucket holding k is size-biased, ~1.1 for s / b = 16; 1.5 is
 // slack); a fused level keeps its window (<= window_frac of it, plus chunk
-// padding).  Levels with at least spec_min_n elements (host estimate) are
-// fused when fused_filter is on; sf_plan[l] is a fused level's sample size.
-// An under-estimate is caught on the device (the final K1 flags
-// "incomplete") and more levels are enqueued.
-int expected_levels(const ss_context* c, u64 n, int b0, int bd, u32 B, bool* spec_plan, int* sf_plan) {
+// padding); a directed level (reading R28: its window is the key bin of the
+// previous fused level's histogram that holds its rank) keeps one of KW_HB
+// bins (4 / KW_HB planned: the bins split the window's key range, not its
+// elements).  Levels with at least spec_min_n elements (host estimate) are
+// fused when fused_filter is on, and the fused levels after the first are
+// directed; sf_plan[l] is a fused level's sample size.  An under-estimate is
+// caught on the device (the final level flags "incomplete") and more levels
+// are enqueued.
+int expected_levels(const ss_context* c, u64 n, int b0, int bd, u32 B, bool* spec_plan, int* sf_plan,
+                    bool* dir_plan) {
     const SpecCfg sp = spec_params(c);
     const double pad = (double)c->sms * 32.0;
     int L = 0;
     double m = (double)n;
+    bool prev_fused = false;
     while (m > (double)B && L < SS_MAX_LEVELS - 2) {
         const int b = L ? bd : b0;
         int sf = fused_sample(c->cfg, L);
-        // (the window's share of the level varies by ~5 % at s = 16384; a
-        // CTA pads half a 32-element chunk on average)
         if (L && c->cfg.sample_size <= 0)
             for (int cand = 4096; cand <= 16384; cand *= 2)
                 if (m * 1.1 * window_frac(sp.z, cand) + pad / 2 <= (double)B) {
@@ -499,10 +503,13 @@ int expected_levels(const ss_context* c, u64 n, int b0, int bd, u32 B, bool* spe
                     break;
                 }
         const double f = window_frac(sp.z, sf);
-        const bool spec = sp.min_n != ~0ull && m >= (double)sp.min_n && f <= sp.max_frac;
+        const bool dir = prev_fused && c->cfg.directed;
+        const bool spec = dir || (sp.min_n != ~0ull && m >= (double)sp.min_n && f <= sp.max_frac);
         if (spec_plan) spec_plan[L] = spec;
         if (sf_plan) sf_plan[L] = sf;
-        m = spec ? m * 1.2 * f + pad : m * 1.5 / b;
+        if (dir_plan) dir_plan[L] = dir;
+        m = dir ? m * 4.0 / KW_HB + pad : spec ? m * 1.2 * f + pad : m * 1.5 / b;
+        prev_fused = spec;
         ++L;
     }
     return L;
@@ -582,6 +589,7 @@ ss_status launch_image(ss_context* c, int H, int lev, int s, int fixup, cudaStre
 struct ExactPlan {
     int b0, bd, s, s_deep;
     int sfs[SS_MAX_LEVELS];           // sample size of each fused level
+    bool dir_plan[SS_MAX_LEVELS];     // level l is directed by level l-1's histogram (R28): no K1w
     u32 B;
     int L;                            // levels [.., L) are enqueued, then the final K1
     bool spec_plan[SS_MAX_LEVELS];    // level l is a fused level
@@ -621,7 +629,7 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
         const int sl = plan_sample(p, lev);
         const int sl_next = lev + 1 < p.L ? plan_sample(p, lev + 1) : 0;
         // a fused level's tail gathers the next level's sample from its output
-        K* pre_next = lev + 1 < p.L && (p.spec_plan[lev + 1] || sl_next <= WIDE_K1_MAX_S)
+        K* pre_next = lev + 1 < p.L && !p.dir_plan[lev + 1] && (p.spec_plan[lev + 1] || sl_next <= WIDE_K1_MAX_S)
                           ? reinterpret_cast<K*>(c->d_presample) + (size_t)(lev + 1) * MAX_S : nullptr;
         const void* pre_this = lev == p.lev_first ? p.sample0
                                : (lev > 0 && p.spec_plan[lev - 1]
@@ -630,7 +638,7 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
         if (p.spec_plan[lev]) {               // fused level: K1w + count/filter in one pass
             const void* pre_buf = pre_this ? pre_this
                                            : (const void*)(reinterpret_cast<K*>(c->d_presample) + (size_t)lev * MAX_S);
-            if ((rc = launch_wsel<T>(c, in, lev, sl, p.B, pre_buf, 0, q))) return rc;
+            if (!p.dir_plan[lev] && (rc = launch_wsel<T>(c, in, lev, sl, p.B, pre_buf, 0, q))) return rc;
             const SpecCfg sp = spec_params(c);
             CountArgs w{};
             w.ctl = c->d_ctl + lev;
@@ -647,6 +655,9 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
             w.seed = (u64)c->cfg.seed;
             w.halt_on_miss = 1;
             w.cap_limit = cap_limit;
+            w.hist = lev + 1 < p.L && p.dir_plan[lev + 1];
+            w.dir_level = p.dir_plan[lev];
+            w.totals = c->d_totals + (size_t)lev * MAX_B;   // the hist bins (zeroed by init)
             mark(c, lev, 1, 0, q);
             if ((rc = launch_window<T>(c, H, in, w, q))) return rc;
             mark(c, lev, 1, 1, q);
@@ -733,7 +744,8 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     c->d2h = 0;
     bool spec_plan[SS_MAX_LEVELS] = {};
     int sf_plan[SS_MAX_LEVELS] = {};
-    int L = expected_levels(c, n, b0, bd, B, spec_plan, sf_plan);
+    bool dir_plan[SS_MAX_LEVELS] = {};
+    int L = expected_levels(c, n, b0, bd, B, spec_plan, sf_plan, dir_plan);
     const int sf = sf_plan[0] ? sf_plan[0] : fused_sample(c->cfg, 0);
     // workspace (reading R16: the paper keeps aux storage <= n/4 elements):
     // the two level buffers hold the planned level-1 survivors with 2x slack
@@ -771,6 +783,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     ExactPlan plan{};
     plan.b0 = b0; plan.bd = bd; plan.s = s; plan.s_deep = s_deep; plan.B = B; plan.L = L;
     std::copy(sf_plan, sf_plan + SS_MAX_LEVELS, plan.sfs);
+    std::copy(dir_plan, dir_plan + SS_MAX_LEVELS, plan.dir_plan);
     std::copy(spec_plan, spec_plan + SS_MAX_LEVELS, plan.spec_plan);
     plan.sample0 = sample0;
     plan.lev_first = 0;
@@ -924,6 +937,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             CK(cudaMemcpyAsync(c->d_ctl + lev_new, c->d_ctl + lh + 1, sizeof(LevelCtl), cudaMemcpyDeviceToDevice, st));
             CK(cudaMemsetAsync(c->d_totals + (size_t)lev_new * MAX_B, 0, sizeof(u64) * MAX_B * (L2 - lev_new + 1), st));
             std::fill(plan.spec_plan, plan.spec_plan + SS_MAX_LEVELS, false);
+            std::fill(plan.dir_plan, plan.dir_plan + SS_MAX_LEVELS, false);
             plan.lev_first = lev_new;
             plan.sample0 = nullptr;
             plan.L = L = L2;

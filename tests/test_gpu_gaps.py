@@ -249,7 +249,11 @@ def test_incomplete_fallback(dtype, cuda_device):
     import paper_conf_ipps_ribizela19_b200 as ss
     c = ss.Context(0, fused_filter=0, b_exact=16, sample_size=256, base_case=256)
     try:
-        n = (1 << 16) + 3
+        # (planned levels: 2^18 -> 24576 -> 2304 -> 216 <= B; after the
+        # poisoned level 0 keeps ~n, two levels of b = 16 leave ~n / 230 > B:
+        # incomplete for any sample of the deeper levels, which are drawn from
+        # the filter's output -- its order is not fixed, reading R15)
+        n = (1 << 18) + 3
         x = _poisoned(n, dtype, 5, c.config["seed"], 256)
         xd = _dev(x)
         seen = 0
