@@ -64,6 +64,7 @@ def parse():
     p.add_argument("--e2e-steps", type=int, default=0, help="host-buffer steps (default: min(steps, 10))")
     p.add_argument("--cpu-seconds", type=float, default=10.0, help="CPU-oracle baseline budget")
     p.add_argument("--no-cpu", action="store_true")
+    p.add_argument("--cfg", default="", help="extra ss_config fields as JSON, e.g. '{\"upper_onepass\": 0}'")
     p.add_argument("--classify", type=int, default=0, help="0 auto (cell LUT where it applies), 1 tree walk")
     p.add_argument("--events", default="separate", choices=["timed", "separate"],
                    help="CUDA events around K2 inside the timed loop (timed: they break the PDL overlap "
@@ -292,6 +293,8 @@ def run_ours(args, rank, world, local_rank):
         ctx.configure(classify=args.classify)
     if not args.fused:
         ctx.configure(fused_filter=0)
+    if args.cfg:
+        ctx.configure(**json.loads(args.cfg))
     upper = args.mode == "upper"
     multi = args.mode == "multi"
     quick = args.mode == "quick"
@@ -444,6 +447,14 @@ def run_ours(args, rank, world, local_rank):
                  "whole call (QuickSelect baseline: per level pivot + partition + decide, SURVEY NEXT-3)")
         k2_bytes = float(last["bytes_algorithmic"])
         tkey = f"{args.mode}_{args.dtype}_2p{args.log2n}"
+    elif upper and last.get("upper_onepass"):
+        # one-pass top-k: level 0 reads the input once, writes its window (the
+        # next level) and streams the keys above it to the output; the bytes
+        # count every key > result as streamed (the few inside the window are
+        # appended by the tail instead: an overcount of at most n_1 elements)
+        kname = "window_kernel (one-pass top-k level 0: count + window copy + keys above the window)"
+        k2_bytes = S * n + S * int(last["n_level"][1]) + S * int(last["upper_greater"])
+        tkey = f"window_upper_{args.dtype}_2p{args.log2n}"
     elif upper:
         kname = "upper_gather_kernel (top-k pass: read the input, write the elements > result)"
         k2_bytes = S * n + S * int(last["upper_greater"])
@@ -460,7 +471,8 @@ def run_ours(args, rank, world, local_rank):
         kname = "count_kernel (K2, level 0)"
         k2_bytes = (S + (1 if exact else 0)) * n          # read S*n, write n oracle bytes
         tkey = f"count_{args.mode}_{args.dtype}_2p{args.log2n}"
-    k2_avg = float(np.mean(upper_ms)) if upper and upper_ms else (ms if multi or quick else kavg(0, 1, prof_timed))
+    up_two = upper and not last.get("upper_onepass")
+    k2_avg = float(np.mean(upper_ms)) if up_two and upper_ms else (ms if multi or quick else kavg(0, 1, prof_timed))
     achieved = k2_bytes / (k2_avg * 1e-3) / 1e9 if k2_avg else 0.0
     traffic = None
     tpath = os.path.join(ROOT, "profiles", "ncu_traffic.json")
@@ -478,6 +490,8 @@ def run_ours(args, rank, world, local_rank):
         "config": {"workload": f"{args.mode} select n=2^{args.log2n} {args.dtype} {args.kind} per GPU, "
                                + _workload_label(args, b, world, last["n_level"]),
                    "n_per_gpu": n, "k": k, "b": b, "kind": args.kind, "fused_filter": args.fused,
+                   **({"ss_config": json.loads(args.cfg)} if args.cfg else {}),
+                   **({"upper_path": "one pass" if last.get("upper_onepass") else "two passes"} if upper else {}),
                    "input_buffers": len(xds),
                    "l2": "inputs larger than L2 (1 GiB input vs 126 MB L2); no flush"
                    if n * S > 2 * L2_BYTES else "WARNING: input fits L2 and is not flushed (use --config)"},

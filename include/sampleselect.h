@@ -37,7 +37,7 @@
 extern "C" {
 #endif
 
-#define SS_ABI_VERSION 6
+#define SS_ABI_VERSION 7
 #define SS_MAX_LEVELS 32
 
 typedef enum { SS_FLOAT32 = 0, SS_FLOAT64 = 1, SS_INT32 = 2, SS_INT64 = 3 } ss_dtype;
@@ -96,6 +96,14 @@ typedef struct {
                              counts the keys it copies in 1024 equal key bins and the bin
                              holding the rank is this level's window (reading R28: exact, no
                              sample, cannot miss); 0 = every fused level draws a sample. */
+    int32_t upper_onepass;/* ss_select_upper: 1 = (default) the top-k fusion of §IV.I in one pass:
+                             a fused level 0 also copies every key above its window to d_out
+                             while it copies the window, and after the select the window's
+                             keys > result and the copies of result complete d_out (no second
+                             read of the input), for outputs n - k <= n / 4; falls back to the
+                             two-pass path when level 0 is not a fused hit.  0 = always two
+                             passes (select, then one threshold pass over the input).  Same
+                             multiset either way. */
 } ss_config;
 
 /* Per-call statistics of the last ss_select / ss_approx_select. */
@@ -139,6 +147,9 @@ typedef struct {
     int64_t workspace_bytes;           /* ss_select: device bytes the context owns after the call
                                           (level buffers sized for the planned survivors; they
                                           grow only when a level would not fit) */
+    int32_t upper_onepass;             /* ss_select_upper: 1 if the one-pass top-k path produced
+                                          d_out (see ss_config.upper_onepass), 0 if two passes ran */
+    int32_t pad_;
 } ss_stats;
 
 /* ---- context --------------------------------------------------------- */

@@ -122,7 +122,8 @@ class Context:
                 "lut_ctas": s.lut_ctas, "upper_greater": s.upper_greater,
                 "ms_upper_gather": s.ms_upper_gather, "ms_quick": s.ms_quick,
                 "incomplete_rounds": s.incomplete_rounds, "shard_levels": s.shard_levels,
-                "shard_ranks": s.shard_ranks, "workspace_bytes": s.workspace_bytes}
+                "shard_ranks": s.shard_ranks, "workspace_bytes": s.workspace_bytes,
+                "upper_onepass": s.upper_onepass}
 
     def raw_tl(self):
         """profile=3: the full 32x3 timeline (us after init; -1 = not stamped)."""

@@ -37,7 +37,8 @@ class SSConfig(ctypes.Structure):
                 ("classify", ctypes.c_int32), ("seed", ctypes.c_uint64),
                 ("fused_filter", ctypes.c_int32), ("spec_z", ctypes.c_float),
                 ("spec_min_n", ctypes.c_int64), ("spec_max_frac", ctypes.c_float),
-                ("shard_gather_log2", ctypes.c_int32), ("directed", ctypes.c_int32)]
+                ("shard_gather_log2", ctypes.c_int32), ("directed", ctypes.c_int32),
+                ("upper_onepass", ctypes.c_int32)]
 
 
 class SSStats(ctypes.Structure):
@@ -54,7 +55,8 @@ class SSStats(ctypes.Structure):
                 ("upper_greater", ctypes.c_int64), ("ms_upper_gather", ctypes.c_float),
                 ("ms_quick", ctypes.c_float), ("incomplete_rounds", ctypes.c_int32),
                 ("shard_levels", ctypes.c_int32), ("shard_ranks", ctypes.c_int32),
-                ("workspace_bytes", ctypes.c_int64)]
+                ("workspace_bytes", ctypes.c_int64), ("upper_onepass", ctypes.c_int32),
+                ("pad_", ctypes.c_int32)]
 
 
 class SSError(RuntimeError):

@@ -80,6 +80,7 @@ ss_status ss_create(int device, ss_context** out) {
     c->cfg.spec_max_frac = 0.25f;
     c->cfg.shard_gather_log2 = 0;
     c->cfg.directed = 1;
+    c->cfg.upper_onepass = 1;
     DevGuard g(device);
     if (cudaDeviceGetAttribute(&c->sms, cudaDevAttrMultiProcessorCount, device) != cudaSuccess) {
         (void)cudaGetLastError();
@@ -117,6 +118,7 @@ void ss_destroy(ss_context* c) {
     cudaFree(c->d_oracles);
     cudaFree(c->d_buf[0]);
     cudaFree(c->d_buf[1]);
+    cudaFree(c->d_win);
     cudaFree(c->d_stage);
     cudaFree(c->d_ctl);
     cudaFree(c->d_res);
@@ -131,6 +133,13 @@ void ss_destroy(ss_context* c) {
     cudaFree(c->d_image);
     cudaFree(c->d_seq);
     cudaFree(c->d_upper_cnt);
+    for (int i = 0; i < MULTI_CH; ++i) {
+        if (c->mchild[i]) ss_destroy(c->mchild[i]);
+        if (c->mchild_st[i]) cudaStreamDestroy(c->mchild_st[i]);
+        if (c->ev_mjoin[i]) cudaEventDestroy(c->ev_mjoin[i]);
+    }
+    if (c->ev_mfork) cudaEventDestroy(c->ev_mfork);
+    if (c->h_mpin) cudaFreeHost(c->h_mpin);
     cudaFree(c->d_multi_scratch);
     cudaFree(c->d_multi);
     cudaFree(c->d_qs);
@@ -190,6 +199,8 @@ ss_status ss_set_config(ss_context* c, const ss_config* cfg) {
         return fail(c, SS_ERR_INVALID_ARGUMENT, "shard_gather_log2 must be 0 or in [12, 28]");
     if (cfg->directed != 0 && cfg->directed != 1)
         return fail(c, SS_ERR_INVALID_ARGUMENT, "directed must be 0 or 1");
+    if (cfg->upper_onepass != 0 && cfg->upper_onepass != 1)
+        return fail(c, SS_ERR_INVALID_ARGUMENT, "upper_onepass must be 0 or 1");
     // captured graphs bake in grid sizes and the fused-filter parameters
     const bool regrid = cfg->ctas_per_sm != c->cfg.ctas_per_sm || cfg->classify != c->cfg.classify ||
                         cfg->fused_filter != c->cfg.fused_filter || cfg->spec_z != c->cfg.spec_z ||

@@ -90,6 +90,9 @@ struct LevelCtl {
     u32 pad3_;
     const void* src;// level 0: the call's input (written by the init kernel, whose argument is patched
                     // per call in a cached CUDA graph); NULL on deeper levels
+    void* up_out;   // level 0 of a top-k call (§IV.I): the caller's output of the n - k largest
+                    // elements (written by the init kernel, patched like src); NULL otherwise
+    u64 ucnt;       // top-k: elements written to up_out so far (the keys above the answer)
 };
 
 struct SelectResult {
@@ -111,6 +114,7 @@ struct SelectResult {
     int halt;                 // level + 1 of a fused level whose window missed rank k (or could not
                               // shrink the level): the chain stopped (done), the host re-runs it
     unsigned long long dist_n;// sharded: the size of the union of the shards (the host plans the next call with it)
+    unsigned long long upper_cnt;// top-k call: #{x > answer} written to the output by the fused path
     int tl_on;                // timeline mode (profile = 3): kernels stamp tl[]
     int pad_;
     u64 t_init;               // %globaltimer at the init kernel (timeline origin)

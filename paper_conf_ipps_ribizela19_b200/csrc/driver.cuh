@@ -36,6 +36,37 @@
 
 using namespace ss;
 
+struct ExactPlan {
+    int b0, bd, s, s_deep;
+    int sfs[SS_MAX_LEVELS];           // sample size of each fused level
+    bool dir_plan[SS_MAX_LEVELS];     // level l is directed by level l-1's histogram (R28): no K1w
+    u32 B;
+    int L;                            // levels [.., L) are enqueued, then the final K1
+    bool spec_plan[SS_MAX_LEVELS];    // level l is a fused level
+    const void* sample0;              // sample keys of level lev_first gathered ahead (or NULL)
+    int lev_first;
+    void* out0;                       // top-k call: level 0 writes its window here (d_win), else NULL
+};
+
+// ss_select_multi: per-rank tails run as exact calls on child contexts, each
+// on its own stream, up to MULTI_CH at a time
+constexpr int MULTI_CH = 8;
+
+// A launched exact call (run_exact_begin) waiting for its result hand-off
+// (run_exact_end): what the host needs for the rare extra rounds.
+struct ExactCall {
+    const void* d;
+    void* up_out;
+    u64 n, k;
+    void* h_result;
+    bool up;
+    int L;
+    u32 B;
+    int b0, bd;
+    double t_in;
+    ExactPlan plan;
+};
+
 struct ss_context {
     int device = 0;
     int sms = 0;
@@ -69,7 +100,8 @@ struct ss_context {
     struct GraphEntry {
         bool used = false;
         int dt = -1;
-        u64 n = 0;
+        u64 sig = 0;                          // the plan's signature (levels, fused / directed flags,
+                                              // sample sizes): n itself is patched like k
         int b0 = 0, bd = 0, s = 0, sd = 0, L = 0, prof = 0;
         u32 B = 0;
         u64 seed = 0;
@@ -80,7 +112,10 @@ struct ss_context {
         void* init_args[16] = {};
         unsigned char init_store[256] = {};   // backing store of the init kernel's arguments
         size_t k_offset = 0;                  // where k lives in init_store
+        size_t n_offset = 0;                  // where n lives in init_store
         size_t d_offset = 0;                  // where the input pointer lives in init_store
+        size_t up_offset = 0;                 // where the top-k output pointer lives (up graphs)
+        bool up = false;                      // top-k graph: level 0 streams the keys above its window
         int kernels = 0;
         u64 stamp = 0;
     } graphs[8];
@@ -107,11 +142,16 @@ struct ss_context {
     unsigned long long* d_upper_cnt = nullptr;  // ss_select_upper: #{x > result}
     cudaEvent_t ev_upper[2] = {nullptr, nullptr};
     unsigned upper_attr = 0;                    // bit dt_code: gather kernel smem attribute set
+    unsigned mf_attr = 0;                       // bit dt_code: multi_filter_kernel smem attribute set
     // ss_select_multi: scratch (sample keys, tree, splitters, eq, totals, search
     // results, bucket counts, one value) and the extracted buckets
     unsigned char* d_multi_scratch = nullptr;
     void* d_multi = nullptr;
     size_t cap_multi = 0;
+    ss_context* mchild[MULTI_CH] = {};          // child contexts of the per-rank tails
+    cudaStream_t mchild_st[MULTI_CH] = {};
+    cudaEvent_t ev_mfork = nullptr, ev_mjoin[MULTI_CH] = {};
+    unsigned char* h_mpin = nullptr;            // pinned staging: ranks in, search rows out, slot tables
     // ss_quickselect: device control block, ping-pong level
     // buffers (level 0 writes up to n - 1 elements), batch-end host mirror
     QsCtl* d_qs = nullptr;
@@ -128,7 +168,13 @@ struct ss_context {
     void* d_gather[2] = {nullptr, nullptr};
     size_t cap_gather[2] = {0, 0};
     int k2_occ[4][11] = {};          // count_kernel<T, H> resident CTAs per SM (per dtype, H)
-    bool kw_attr[4][2] = {};         // window_kernel<T, APX> shared-memory attribute set
+    bool kw_attr[4][3] = {};         // window_kernel<T, APX, UP> shared-memory attribute set
+    // ss_select_upper one-pass path: level 0's window, kept for the top-k tail
+    // (level 1 reads it; deeper levels ping-pong in d_buf)
+    void* d_win = nullptr;
+    size_t cap_win = 0;
+    bool up_used = false;            // the last run_exact ran the one-pass top-k path
+    ExactCall call{};                // the exact call in flight (run_exact_begin .. run_exact_end)
     bool host_timing = false;
     double ht[5] = {};
     long long ht_n = 0;
@@ -292,16 +338,16 @@ ss_status launch_count(ss_context* c, int H, const T* in, CountArgs& a, cudaStre
 }
 
 // fused count + filter kernel: one CTA per SM, KW_SMEM bytes (TMA ring + stash)
-template <typename T, bool APX = false>
+template <typename T, bool APX = false, bool UP = false>
 ss_status launch_window(ss_context* c, int /*H*/, const T* in, CountArgs a, cudaStream_t st) {
     a.grid = (u32)c->sms * (u32)KW_MINB;
-    bool& attr_set = c->kw_attr[dt_code<T>() - 1][APX ? 1 : 0];
+    bool& attr_set = c->kw_attr[dt_code<T>() - 1][APX ? 1 : UP ? 2 : 0];
     if (!attr_set) {
-        CK(cudaFuncSetAttribute(window_kernel<T, APX>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+        CK(cudaFuncSetAttribute(window_kernel<T, APX, UP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 (int)KW_SMEM));
         attr_set = true;
     }
-    CK(launch_pdl(window_kernel<T, APX>, dim3(a.grid), dim3(KW_THREADS), KW_SMEM, st, in, a));
+    CK(launch_pdl(window_kernel<T, APX, UP>, dim3(a.grid), dim3(KW_THREADS), KW_SMEM, st, in, a));
     CKLAUNCH("window_kernel");
     return SS_OK;
 }
@@ -586,16 +632,12 @@ ss_status launch_image(ss_context* c, int H, int lev, int s, int fixup, cudaStre
 // ends with the final K1 (base case, or the "incomplete" flag when an unlucky
 // sample left more than B elements).  Level p.lev_first reads `first_in`;
 // level l > p.lev_first reads the buffer level l-1 wrote (d_buf[(l-1) & 1]).
-struct ExactPlan {
-    int b0, bd, s, s_deep;
-    int sfs[SS_MAX_LEVELS];           // sample size of each fused level
-    bool dir_plan[SS_MAX_LEVELS];     // level l is directed by level l-1's histogram (R28): no K1w
-    u32 B;
-    int L;                            // levels [.., L) are enqueued, then the final K1
-    bool spec_plan[SS_MAX_LEVELS];    // level l is a fused level
-    const void* sample0;              // sample keys of level lev_first gathered ahead (or NULL)
-    int lev_first;
-};
+
+
+// The buffer level `lev` writes (and level lev + 1 reads).
+inline void* level_out(const ss_context* c, const ExactPlan& p, int lev) {
+    return lev == 0 && p.out0 ? p.out0 : c->d_buf[lev & 1];
+}
 
 inline int plan_sample(const ExactPlan& p, int lev) {
     if (p.spec_plan[lev]) return p.sfs[lev];
@@ -621,8 +663,9 @@ template <typename T>
 ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first_in, int lev0, cudaStream_t q) {
     typedef typename Traits<T>::Key K;
     ss_status rc;
-    const T* in = lev0 > p.lev_first ? reinterpret_cast<const T*>(c->d_buf[(lev0 - 1) & 1]) : first_in;
-    const u64 cap_limit = std::min(c->cap_buf[0], c->cap_buf[1]) / sizeof(T);   // elements per level buffer
+    const T* in = lev0 > p.lev_first ? reinterpret_cast<const T*>(level_out(c, p, lev0 - 1)) : first_in;
+    const u64 cap_limit = std::min(std::min(c->cap_buf[0], c->cap_buf[1]), p.out0 ? c->cap_win : ~(size_t)0) /
+                          sizeof(T);          // elements per level buffer
     int lev = lev0;
     for (; lev < p.L; ++lev) {
         const int b = lev ? p.bd : p.b0, H = log2i(b);
@@ -646,7 +689,7 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
             w.res = c->d_res;
             w.level = lev;
             w.tail = TAIL_EXACT;
-            w.cap_out = c->d_buf[lev & 1];    // the window = the next level's input
+            w.cap_out = level_out(c, p, lev);  // the window = the next level's input
             w.spec_min_n = sp.min_n;
             w.spec_z = sp.z;
             w.spec_max_frac = sp.max_frac;
@@ -659,10 +702,14 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
             w.dir_level = p.dir_plan[lev];
             w.totals = c->d_totals + (size_t)lev * MAX_B;   // the hist bins (zeroed by init)
             mark(c, lev, 1, 0, q);
-            if ((rc = launch_window<T>(c, H, in, w, q))) return rc;
+            if (lev == 0 && p.out0) {          // top-k: also stream the keys above the window out
+                if ((rc = launch_window<T, false, true>(c, H, in, w, q))) return rc;
+            } else if ((rc = launch_window<T>(c, H, in, w, q))) {
+                return rc;
+            }
             mark(c, lev, 1, 1, q);
             ++c->launches;
-            in = reinterpret_cast<const T*>(c->d_buf[lev & 1]);
+            in = reinterpret_cast<const T*>(level_out(c, p, lev));
             continue;
         }
         const u32 grid = grid_for<T>(c, H);
@@ -705,7 +752,7 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
         mark(c, lev, 1, 1, q);
         ++c->launches;
         if (a.grid != grid) return fail(c, SS_ERR_INTERNAL, "grid mismatch");
-        T* out = reinterpret_cast<T*>(c->d_buf[lev & 1]);
+        T* out = reinterpret_cast<T*>(level_out(c, p, lev));
         FilterArgs f{};
         f.ctl = c->d_ctl + lev;
         f.res = c->d_res;
@@ -725,8 +772,27 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
     return launch_wsel<T>(c, in, lev, 0, p.B, nullptr, 1, q);
 }
 
+// top-k tail: the window's keys above the answer, then the copies of it
 template <typename T>
-ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cudaStream_t st) {
+ss_status enqueue_upper_tail(ss_context* c, bool up, cudaStream_t q) {
+    if (!up) return SS_OK;
+    CK(launch_pdl(upper_window_kernel<T>, dim3((u32)c->sms * 2), dim3(UW_THREADS), 0, q,
+                  reinterpret_cast<const T*>(c->d_win), c->d_ctl, (const SelectResult*)c->d_res));
+    CKLAUNCH("upper_window_kernel");
+    CK(launch_pdl(upper_tail_fill_kernel<T>, dim3((u32)c->sms * 4), dim3(256), 0, q, c->d_ctl, c->d_res));
+    CKLAUNCH("upper_tail_fill_kernel");
+    c->launches += 2;
+    return SS_OK;
+}
+
+// An exact call in two halves: run_exact_begin plans it and launches the
+// planned chain (one graph launch) without waiting; run_exact_end waits for the
+// result hand-off, runs the rare extra rounds and fills the stats.  Callers
+// with independent selects (ss_select_multi) launch several on their own
+// contexts and streams before waiting on any.
+template <typename T>
+ss_status run_exact_begin(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cudaStream_t st,
+                          T* up_out = nullptr) {
     typedef typename Traits<T>::Key K;
     const double t_in = c->host_timing ? now_us() : 0.0;
     // reading R7: level 0 draws s = clamp(16 b, 4096, 16384) samples (or the
@@ -747,6 +813,10 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     bool dir_plan[SS_MAX_LEVELS] = {};
     int L = expected_levels(c, n, b0, bd, B, spec_plan, sf_plan, dir_plan);
     const int sf = sf_plan[0] ? sf_plan[0] : fused_sample(c->cfg, 0);
+    // top-k (§IV.I): a fused level 0 also streams the keys above its window to
+    // up_out and keeps its window in d_win for the tail kernels
+    const bool up = up_out && L > 0 && spec_plan[0];
+    c->up_used = up;
     // workspace (reading R16: the paper keeps aux storage <= n/4 elements):
     // the two level buffers hold the planned level-1 survivors with 2x slack
     // (a level whose survivors would not fit halts before writing past them;
@@ -759,6 +829,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
         const u64 cap_el = std::min<u64>(n, std::max<u64>((u64)(2.0 * est1), (u64)1 << 20));
         for (int i = 0; i < 2; ++i)
             if ((rc = grow(c, &c->d_buf[i], &c->cap_buf[i], cap_el * sizeof(T)))) return rc;
+        if (up && (rc = grow(c, &c->d_win, &c->cap_win, cap_el * sizeof(T)))) return rc;
         bool paper_deep = false;
         for (int l = 1; l < L; ++l) paper_deep |= !spec_plan[l];
         const u64 orc = L > 0 && !spec_plan[0] ? n : paper_deep ? cap_el : 0;
@@ -775,7 +846,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     auto enqueue_init = [&](cudaStream_t q) -> ss_status {
         CK(launch_pdl(init_kernel<T>, dim3(pre0 ? ((u32)s_init + 255u) / 256u : 1u), dim3(256), 0, q, c->d_ctl,
                       (int)(SS_MAX_LEVELS + 1), c->d_totals, (int)((L + 1) * MAX_B), c->d_res, n, k, tl_on, d,
-                      s_init, (u64)c->cfg.seed, sample0));
+                      s_init, (u64)c->cfg.seed, sample0, up ? (void*)up_out : nullptr));
         CKLAUNCH("init_kernel");
         ++c->launches;
         return SS_OK;
@@ -787,19 +858,31 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     std::copy(spec_plan, spec_plan + SS_MAX_LEVELS, plan.spec_plan);
     plan.sample0 = sample0;
     plan.lev_first = 0;
+    plan.out0 = up ? c->d_win : nullptr;
     auto enqueue_levels = [&](int lev0, cudaStream_t q) -> ss_status {
         plan.L = L;
         return enqueue_exact_levels<T>(c, plan, d, lev0, q);
     };
     // the planned part of the call: one CUDA graph launch (events of
-    // profile 1/2 cannot live in a graph: those calls launch directly)
+    // profile 1/2 cannot live in a graph: those calls launch directly).  The
+    // chain depends on n only through the plan (every kernel reads its level's
+    // size from the LevelCtl): graphs are keyed on the plan's signature and
+    // n, k, the input and output pointers are patched into the init node.
     const bool graph = c->use_graphs && c->cfg.profile != 1 && c->cfg.profile != 2;
     ss_context::GraphEntry* ge = nullptr;
+    u64 sig = 1469598103934665603ull;
+    {
+        auto mix = [&](u64 v) { sig = (sig ^ v) * 1099511628211ull; };
+        mix((u64)L);
+        mix((u64)s_init);
+        mix((u64)pre0);
+        for (int l = 0; l < L; ++l) mix((u64)spec_plan[l] | (u64)dir_plan[l] << 1 | (u64)(u32)sf_plan[l] << 2);
+    }
     if (graph) {
         for (auto& e : c->graphs)
             if (e.used && e.dt == dt_code<T>() &&
-                e.n == n && e.b0 == b0 && e.bd == bd && e.s == s && e.sd == s_deep && e.L == L &&
-                e.prof == tl_on && e.B == B && e.seed == c->cfg.seed)
+                e.sig == sig && e.b0 == b0 && e.bd == bd && e.s == s && e.sd == s_deep && e.L == L &&
+                e.prof == tl_on && e.B == B && e.seed == c->cfg.seed && e.up == up)
                 ge = &e;
         if (!ge) {
             ss_context::GraphEntry* slot = nullptr;           // a free entry, else the least recently used
@@ -817,6 +900,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             CK(cudaStreamBeginCapture(c->cap_st, cudaStreamCaptureModeThreadLocal));
             ss_status rc2 = enqueue_init(c->cap_st);
             if (!rc2) rc2 = enqueue_levels(0, c->cap_st);
+            if (!rc2) rc2 = enqueue_upper_tail<T>(c, up, c->cap_st);
             if (!rc2) rc2 = enqueue_publish(c, c->cap_st);
             cudaGraph_t g = nullptr;
             const cudaError_t ec = cudaStreamEndCapture(c->cap_st, &g);
@@ -853,24 +937,26 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             }
             slot->used = true;
             slot->dt = dt_code<T>();
-            slot->n = n;
+            slot->sig = sig;
             slot->b0 = b0; slot->bd = bd; slot->s = s; slot->sd = s_deep; slot->L = L;
-            slot->prof = tl_on; slot->B = B; slot->seed = c->cfg.seed;
+            slot->prof = tl_on; slot->B = B; slot->seed = c->cfg.seed; slot->up = up;
             slot->exec = ex;
             slot->init_node = init_node;
             slot->kernels = c->launches - launches0;
             // private copy of the init arguments; k is the 7th (index 6)
             slot->init_params = ip;
             size_t off = 0;
-            const size_t sizes[12] = {sizeof(LevelCtl*), sizeof(int), sizeof(u64*), sizeof(int), sizeof(SelectResult*),
+            const size_t sizes[13] = {sizeof(LevelCtl*), sizeof(int), sizeof(u64*), sizeof(int), sizeof(SelectResult*),
                                       sizeof(u64), sizeof(u64), sizeof(int), sizeof(const T*), sizeof(int), sizeof(u64),
-                                      sizeof(K*)};
-            for (int i = 0; i < 12; ++i) {
+                                      sizeof(K*), sizeof(void*)};
+            for (int i = 0; i < 13; ++i) {
                 off = (off + 7) & ~(size_t)7;
                 std::memcpy(slot->init_store + off, ip.kernelParams[i], sizes[i]);
                 slot->init_args[i] = slot->init_store + off;
+                if (i == 5) slot->n_offset = off;
                 if (i == 6) slot->k_offset = off;
                 if (i == 8) slot->d_offset = off;
+                if (i == 12) slot->up_offset = off;
                 off += sizes[i];
             }
             slot->init_params.kernelParams = slot->init_args;
@@ -882,12 +968,17 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             // the rank and the input pointer are arguments of the init kernel
             // only (later kernels read level 0's input from LevelCtl::src):
             // patch them into the cached graph
-            u64 kk = k;
+            u64 kk = k, nn = n;
             const T* dd = d;
+            void* uo = up ? (void*)up_out : nullptr;
             if (std::memcmp(ge->init_store + ge->k_offset, &kk, sizeof(u64)) ||
-                std::memcmp(ge->init_store + ge->d_offset, &dd, sizeof(const T*))) {   // (unchanged: no update)
+                std::memcmp(ge->init_store + ge->n_offset, &nn, sizeof(u64)) ||
+                std::memcmp(ge->init_store + ge->d_offset, &dd, sizeof(const T*)) ||
+                std::memcmp(ge->init_store + ge->up_offset, &uo, sizeof(void*))) {   // (unchanged: no update)
                 std::memcpy(ge->init_store + ge->k_offset, &kk, sizeof(u64));
+                std::memcpy(ge->init_store + ge->n_offset, &nn, sizeof(u64));
                 std::memcpy(ge->init_store + ge->d_offset, &dd, sizeof(const T*));
+                std::memcpy(ge->init_store + ge->up_offset, &uo, sizeof(void*));
                 CK(cudaGraphExecKernelNodeSetParams(ge->exec, ge->init_node, &ge->init_params));
             }
         }
@@ -900,8 +991,41 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
     } else {
         if ((rc = enqueue_init(st))) return rc;
         if ((rc = enqueue_levels(0, st))) return rc;
+        if ((rc = enqueue_upper_tail<T>(c, up, st))) return rc;
         if ((rc = enqueue_publish(c, st))) return rc;
     }
+    ExactCall& ec = c->call;
+    ec.d = d;
+    ec.up_out = up_out;
+    ec.n = n;
+    ec.k = k;
+    ec.h_result = h_result;
+    ec.up = up;
+    ec.L = L;
+    ec.B = B;
+    ec.b0 = b0;
+    ec.bd = bd;
+    ec.t_in = t_in;
+    ec.plan = plan;
+    return SS_OK;
+}
+
+template <typename T>
+ss_status run_exact_end(ss_context* c, cudaStream_t st) {
+    ExactCall& ec = c->call;
+    const T* d = reinterpret_cast<const T*>(ec.d);
+    const u64 n = ec.n;
+    const bool up = ec.up;
+    int L = ec.L;
+    const u32 B = ec.B;
+    const int b0 = ec.b0, bd = ec.bd;
+    const double t_in = ec.t_in;
+    ExactPlan& plan = ec.plan;
+    ss_status rc;
+    auto enqueue_levels = [&](int lev0, cudaStream_t q) -> ss_status {
+        plan.L = L;
+        return enqueue_exact_levels<T>(c, plan, d, lev0, q);
+    };
     const double t_w = c->host_timing ? now_us() : 0.0;
     if ((rc = wait_publish(c, st))) return rc;
     if (c->host_timing) c->ht[2] += now_us() - t_w;
@@ -923,6 +1047,9 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
                 const int bi = (lh - 1) & 1;
                 if ((rc = grow_keep(c, &c->d_buf[bi], &c->cap_buf[bi], n * sizeof(T), lh ? keep : 0, st))) return rc;
                 if ((rc = grow_keep(c, &c->d_buf[bi ^ 1], &c->cap_buf[bi ^ 1], n * sizeof(T), 0, st))) return rc;
+                if (up && (rc = grow_keep(c, &c->d_win, &c->cap_win, n * sizeof(T), lh == 1 ? keep : 0, st)))
+                    return rc;
+                if (up) plan.out0 = c->d_win;
             }
             if ((rc = grow(c, (void**)&c->d_oracles, &c->cap_oracles, nh + 64))) return rc;
             double m = (double)nh;
@@ -941,7 +1068,7 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
             plan.lev_first = lev_new;
             plan.sample0 = nullptr;
             plan.L = L = L2;
-            const T* first_in = lh == 0 ? d : reinterpret_cast<const T*>(c->d_buf[(lh - 1) & 1]);
+            const T* first_in = lh == 0 ? d : reinterpret_cast<const T*>(level_out(c, plan, lh - 1));
             if ((rc = enqueue_exact_levels<T>(c, plan, first_in, lev_new, st))) return rc;
         } else if (!h.done) {
             ++extra_rounds;
@@ -958,8 +1085,13 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
         if ((rc = enqueue_publish(c, st))) return rc;
         if ((rc = wait_publish(c, st))) return rc;
     }
+    if (up && extra_rounds) {                  // the tail kernels of the graph saw an unfinished call
+        if ((rc = enqueue_upper_tail<T>(c, up, st))) return rc;
+        if ((rc = enqueue_publish(c, st))) return rc;
+        if ((rc = wait_publish(c, st))) return rc;
+    }
     const SelectResult& r = *c->h_res;
-    std::memcpy(h_result, &r.bits, sizeof(T));
+    std::memcpy(ec.h_result, &r.bits, sizeof(T));
     ss_stats& S = c->stats;
     std::memset(&S, 0, sizeof(S));
     S.levels = r.levels;
@@ -1005,6 +1137,12 @@ ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cud
 }
 
 template <typename T>
+ss_status run_exact(ss_context* c, const T* d, u64 n, u64 k, void* h_result, cudaStream_t st, T* up_out = nullptr) {
+    const ss_status rc = run_exact_begin<T>(c, d, n, k, h_result, st, up_out);
+    return rc ? rc : run_exact_end<T>(c, st);
+}
+
+template <typename T>
 ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_result, int64_t* h_rank,
                      cudaStream_t st) {
     typedef typename Traits<T>::Key K;
@@ -1020,7 +1158,7 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     const bool wide = s <= WIDE_K1_MAX_S || merge;
     K* sample0 = s <= WIDE_K1_MAX_S ? reinterpret_cast<K*>(c->d_sample0) : nullptr;
     CK(launch_pdl(init_kernel<T>, dim3(sample0 ? ((u32)s + 255u) / 256u : 1u), dim3(256), 0, st, c->d_ctl, 2, c->d_totals,
-                  (int)MAX_B, c->d_res, n, k, (int)(c->cfg.profile == 3), d, s, (u64)c->cfg.seed, sample0));
+                  (int)MAX_B, c->d_res, n, k, (int)(c->cfg.profile == 3), d, s, (u64)c->cfg.seed, sample0, (void*)nullptr));
     CKLAUNCH("init_kernel");
     ++c->launches;
     // fused one-pass window (approx_window in kernels.cuh) on large inputs;
@@ -1120,14 +1258,43 @@ ss_status launch_ablation(ss_context* c, const T* d, u64 n, const void* tree, in
     return SS_OK;
 }
 
-// Top-k fusion (§IV.I; reading R22): the exact select, then one
-// streaming pass that appends the elements > result to d_out, then the
-// copies of result that fill it up to n-k.
+// Top-k fusion (§IV.I; reading R22).  One pass (upper_onepass, the
+// paper's design: the filter "copies not only elements from the target
+// bucket, but also from all buckets containing larger elements"): the fused
+// level 0 streams the keys above its window straight to d_out while it copies
+// the window; the select finishes on the window, and the tail kernels append
+// the window's keys > result and the copies of result -- all inside the call's
+// graph.  Otherwise (level 0 not a fused hit, or upper_onepass = 0): the exact
+// select, then one streaming pass that appends the elements > result to d_out,
+// then the copies of result that fill it up to n-k.
+#ifndef SS_UPPER_ONEPASS_MAX_FRAC
+#define SS_UPPER_ONEPASS_MAX_FRAC 0.25
+#endif
+constexpr double UPPER_ONEPASS_MAX_FRAC = SS_UPPER_ONEPASS_MAX_FRAC;
 template <typename T>
 ss_status run_upper(ss_context* c, const T* d, u64 n, u64 k, T* d_out, void* h_result, cudaStream_t st) {
     typedef typename Traits<T>::Key K;
-    ss_status rc = run_exact<T>(c, d, n, k, h_result, st);
+    // the one-pass path appends the keys above level 0's window with one
+    // global atomic per warp flush: measured at n = 2^28 fp32 it wins while
+    // the output is small and loses to the two passes (select + a streaming
+    // gather with CTA-staged appends) once n - k is a large part of n
+    const bool one = c->cfg.upper_onepass && (double)(n - k) <= UPPER_ONEPASS_MAX_FRAC * (double)n;
+    ss_status rc = run_exact<T>(c, d, n, k, h_result, st, one ? d_out : nullptr);
     if (rc) return rc;
+    const u64 m = n - k;
+    {
+        const SelectResult& r = *c->h_res;
+        const bool l0_ok = (r.spec_levels & 1) && ((r.fused_levels & 1) || (r.eq_exit && r.levels == 1));
+        if (c->up_used && l0_ok) {
+            const u64 greater = r.upper_cnt;
+            if (greater >= m && m > 0) return fail(c, SS_ERR_INTERNAL, "select_upper: #{x > result} >= n-k");
+            c->stats.upper_greater = (int64_t)greater;
+            c->stats.upper_onepass = 1;
+            // + the output, + the tail's read of level 0's window
+            c->stats.bytes_algorithmic += (double)sizeof(T) * ((double)m + (double)r.n_level[1] * (r.fused_levels & 1));
+            return SS_OK;
+        }
+    }
     if (!c->d_upper_cnt) CK(cudaMalloc(&c->d_upper_cnt, sizeof(unsigned long long)));
     const bool prof = c->cfg.profile != 0;
     if (prof && !c->ev_upper[0]) {
@@ -1139,7 +1306,6 @@ ss_status run_upper(ss_context* c, const T* d, u64 n, u64 k, T* d_out, void* h_r
     K vb;
     std::memcpy(&vb, &v, sizeof(T));
     const K kv = Traits<T>::to_key(vb);
-    const u64 m = n - k;
     CK(cudaMemsetAsync(c->d_upper_cnt, 0, sizeof(unsigned long long), st));
     constexpr u64 EPV = 16 / sizeof(T);
     const u64 tiles = (n / EPV + (u64)UG_THREADS * UG_VEC - 1) / ((u64)UG_THREADS * UG_VEC);
@@ -1173,17 +1339,39 @@ ss_status run_upper(ss_context* c, const T* d, u64 n, u64 k, T* d_out, void* h_r
 
 // Multi-rank selection (§VI "multiple ... selection",
 // reading R23): m ranks share one sample, one splitter tree and ONE count
-// pass over the input (the dominant K2 pass, §IV.G); every distinct bucket
-// holding a rank is extracted once (K5, all extractions before any deeper
-// level because the deeper levels reuse the oracle bytes), and each rank then
+// pass over the input (the dominant K2 pass, §IV.G); one launch searches the
+// bucket of every rank; every distinct bucket holding a rank is extracted in
+// one pass over the oracle bytes (multi_filter_kernel); each rank then
 // finishes with the single-rank select on its bucket (rank k - r_j, Fig. 1).
-// An equality bucket answers its ranks with its splitter (§IV.C).
+// An equality bucket answers its ranks with its splitter (§IV.C).  One host
+// round trip (the search rows, which size the extraction); the per-rank
+// selects run as exact calls on child contexts, each on its own stream, all
+// launched (one graph launch each) before the host waits on any.
 constexpr int MULTI_MAX = 1024;
 constexpr u64 MULTI_MIN_N = (u64)1 << 20;   // below: one select per rank is cheaper
-// Below 4 ranks the per-rank fused selects win: measured at n = 2^28 fp32
-// (profiles/r01f_bench_multi1.json, profiles/r01f_bench_multi8.json) the shared
-// path costs ~0.50 ms + ~0.18 ms per extra rank, a fused single select 0.28 ms.
+// Below 4 ranks the per-rank fused selects win: each is one ~0.22 ms pass at
+// n = 2^28 fp32, the shared path's count + extraction alone ~0.33 ms.
 constexpr int MULTI_MIN_M = 4;
+
+// the child contexts (same device and config, no profiling) and their streams
+inline ss_status multi_children(ss_context* c, int want) {
+    if (!c->ev_mfork) CK(cudaEventCreateWithFlags(&c->ev_mfork, cudaEventDisableTiming));
+    ss_config cc = c->cfg;
+    cc.profile = 0;
+    for (int i = 0; i < want && i < MULTI_CH; ++i) {
+        if (!c->mchild[i]) {
+            ss_status rc = ss_create(c->device, &c->mchild[i]);
+            if (rc) return fail(c, rc, "select_multi: child context");
+            CK(cudaStreamCreateWithFlags(&c->mchild_st[i], cudaStreamNonBlocking));
+            CK(cudaEventCreateWithFlags(&c->ev_mjoin[i], cudaEventDisableTiming));
+        }
+        if (std::memcmp(&c->mchild[i]->cfg, &cc, sizeof(cc))) {
+            ss_status rc = ss_set_config(c->mchild[i], &cc);
+            if (rc) return fail(c, rc, c->mchild[i]->err.c_str());
+        }
+    }
+    return SS_OK;
+}
 
 template <typename T>
 ss_status run_multi(ss_context* c, ss_dtype dt, const T* d, u64 n, int m, const int64_t* ks, void* h_res,
@@ -1205,100 +1393,127 @@ ss_status run_multi(ss_context* c, ss_dtype dt, const T* d, u64 n, int m, const 
     }
     const int b = std::min(c->cfg.b_exact, 256);
     const int s = c->cfg.sample_size > 0 ? c->cfg.sample_size : sample_size(c->cfg, b);
-    // scratch layout (8-byte slots)
+    // device scratch layout (8-byte slots)
     const size_t o_keys = 0, o_tree = o_keys + (size_t)MAX_S * 8, o_spl = o_tree + (size_t)MAX_B * 8,
                  o_tot = o_spl + (size_t)MAX_B * 8, o_srch = o_tot + (size_t)MAX_B * 8,
-                 o_cnt = o_srch + (size_t)MULTI_MAX * 32, o_val = o_cnt + (size_t)MULTI_MAX * 8,
-                 o_eq = o_val + 64, o_lut = o_eq + MAX_B, o_sb = o_lut + 256,
+                 o_ks = o_srch + (size_t)MULTI_MAX * MS_ROW * 8, o_cnt = o_ks + (size_t)MULTI_MAX * 8,
+                 o_eq = o_cnt + (size_t)MULTI_MAX * 8, o_lut = o_eq + MAX_B, o_sb = o_lut + 256,
                  o_sbase = o_sb + (size_t)MF_MAX_SLOTS * 4, scratch = o_sbase + (size_t)MF_MAX_SLOTS * 8;
+    // pinned host staging (ranks, search rows, slot tables): the copies stay asynchronous
+    const size_t p_ks = 0, p_srch = p_ks + (size_t)MULTI_MAX * 8, p_lut = p_srch + (size_t)MULTI_MAX * MS_ROW * 8,
+                 p_sb = p_lut + 256, p_sbase = p_sb + (size_t)MF_MAX_SLOTS * 4,
+                 pin_bytes = p_sbase + (size_t)MF_MAX_SLOTS * 8;
     if (!c->d_multi_scratch) CK(cudaMalloc(&c->d_multi_scratch, scratch));
+    if (!c->h_mpin) CK(cudaMallocHost(&c->h_mpin, pin_bytes));
     unsigned char* S0 = c->d_multi_scratch;
+    unsigned char* P0 = c->h_mpin;
     if ((rc = ensure_small(c))) return rc;
     if ((rc = grow(c, (void**)&c->d_oracles, &c->cap_oracles, (size_t)n + 64))) return rc;
+    std::memcpy(P0 + p_ks, ks, sizeof(int64_t) * (size_t)m);
+    CK(cudaMemcpyAsync(S0 + o_ks, P0 + p_ks, sizeof(int64_t) * (size_t)m, cudaMemcpyHostToDevice, st));
     if ((rc = ss_step_sample(c, dt, d, (int64_t)n, 0, 0, s, S0 + o_keys, st))) return rc;
     if ((rc = ss_step_tree(c, dt, S0 + o_keys, s, b, 1, S0 + o_tree, S0 + o_spl, S0 + o_eq, st))) return rc;
     if ((rc = ss_step_count(c, dt, d, (int64_t)n, S0 + o_tree, b, (uint64_t*)(S0 + o_tot), c->d_oracles, st)))
         return rc;
-    for (int i = 0; i < m; ++i)
-        if ((rc = ss_step_search(c, (const uint64_t*)(S0 + o_tot), b, ks[i], S0 + o_eq,
-                                 (int64_t*)(S0 + o_srch) + 4 * (size_t)i, st)))
-            return rc;
-    std::vector<int64_t> sr((size_t)m * 4);
-    CK(cudaMemcpyAsync(sr.data(), S0 + o_srch, sizeof(int64_t) * 4 * (size_t)m, cudaMemcpyDeviceToHost, st));
-    CK(cudaStreamSynchronize(st));
-    int step_launches = 3 + m;
+    multi_search_kernel<T><<<1, 256, 0, st>>>((const u64*)(S0 + o_tot), (u32)b, (const long long*)(S0 + o_ks), m,
+                                               S0 + o_eq, (const K*)(S0 + o_spl), (long long*)(S0 + o_srch));
+    CK(cudaGetLastError());
+    const int64_t* sr = reinterpret_cast<const int64_t*>(P0 + p_srch);
+    CK(cudaMemcpyAsync(P0 + p_srch, S0 + o_srch, sizeof(int64_t) * MS_ROW * (size_t)m, cudaMemcpyDeviceToHost, st));
+    CK(cudaStreamSynchronize(st));             // the one host round trip: the rows size the extraction
+    int step_launches = 4;
     bytes += (double)sizeof(T) * n + (double)n;   // count: read + oracle bytes
     // distinct buckets, in bucket order; regions of d_multi for the non-equality ones
     std::vector<int> order(m);
     for (int i = 0; i < m; ++i) order[i] = i;
-    std::sort(order.begin(), order.end(), [&](int a, int bb) { return sr[4 * (size_t)a] < sr[4 * (size_t)bb]; });
+    std::sort(order.begin(), order.end(),
+              [&](int a, int bb) { return sr[MS_ROW * (size_t)a] < sr[MS_ROW * (size_t)bb]; });
     std::vector<int64_t> bucket_off(MAX_B, -1);
     size_t total = 0;
     for (int i : order) {
-        const int64_t j = sr[4 * (size_t)i], nj = sr[4 * (size_t)i + 2], eq = sr[4 * (size_t)i + 3];
+        const int64_t j = sr[MS_ROW * (size_t)i], nj = sr[MS_ROW * (size_t)i + 2], eq = sr[MS_ROW * (size_t)i + 3];
         if (eq || bucket_off[j] >= 0) continue;
         bucket_off[j] = (int64_t)total;
         total += (size_t)nj;
     }
     if ((rc = grow(c, &c->d_multi, &c->cap_multi, std::max<size_t>(total, 1) * sizeof(T)))) return rc;
-    std::vector<u32> slot_bucket;
-    std::vector<u64> slot_base;
+    u32* slot_bucket = reinterpret_cast<u32*>(P0 + p_sb);
+    u64* slot_base = reinterpret_cast<u64*>(P0 + p_sbase);
+    int nb = 0;
     for (int j = 0; j < b; ++j)
         if (bucket_off[j] >= 0) {
-            slot_bucket.push_back((u32)j);
-            slot_base.push_back((u64)bucket_off[j]);
+            if (nb < MF_MAX_SLOTS) {
+                slot_bucket[nb] = (u32)j;
+                slot_base[nb] = (u64)bucket_off[j];
+            }
+            ++nb;
         }
-    const int nb = (int)slot_bucket.size();
     if (nb >= 2 && nb <= MF_MAX_SLOTS && b <= 256) {
         // one pass over the oracle bytes extracts every wanted bucket
-        std::vector<uint8_t> slot_of(256, 0xFF);
+        uint8_t* slot_of = P0 + p_lut;
+        std::memset(slot_of, 0xFF, 256);
         for (int i = 0; i < nb; ++i) slot_of[slot_bucket[i]] = (uint8_t)i;
-        CK(cudaMemcpyAsync(S0 + o_lut, slot_of.data(), 256, cudaMemcpyHostToDevice, st));
-        CK(cudaMemcpyAsync(S0 + o_sb, slot_bucket.data(), sizeof(u32) * nb, cudaMemcpyHostToDevice, st));
-        CK(cudaMemcpyAsync(S0 + o_sbase, slot_base.data(), sizeof(u64) * nb, cudaMemcpyHostToDevice, st));
-        multi_filter_kernel<T><<<c->step_grid, MF_THREADS, 0, st>>>(
+        CK(cudaMemcpyAsync(S0 + o_lut, P0 + p_lut, 256 + (size_t)MF_MAX_SLOTS * 12, cudaMemcpyHostToDevice, st));
+        if (!(c->mf_attr >> dt_code<T>() & 1)) {
+            CK(cudaFuncSetAttribute(multi_filter_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)MF_SMEM));
+            c->mf_attr |= 1u << dt_code<T>();
+        }
+        multi_filter_kernel<T><<<c->step_grid, MF_THREADS, MF_SMEM, st>>>(
             d, n, c->d_oracles, c->d_cta_counts, (u32)b, c->step_grid, S0 + o_lut, (const u32*)(S0 + o_sb),
             (const u64*)(S0 + o_sbase), (u32)nb, (T*)c->d_multi);
         CK(cudaGetLastError());
         step_launches += 1;
         bytes += (double)n;    // one read of the oracle bytes
-        CK(cudaStreamSynchronize(st));   // the host slot vectors go out of scope
     } else {
-        for (int i = 0; i < nb; ++i) {
-            if ((rc = ss_step_filter(c, dt, d, (int64_t)n, c->d_oracles, (int32_t)slot_bucket[i],
-                                     (T*)c->d_multi + slot_base[i], (uint64_t*)(S0 + o_cnt) + i, st)))
+        for (int j = 0; j < b; ++j) {
+            if (bucket_off[j] < 0) continue;
+            if ((rc = ss_step_filter(c, dt, d, (int64_t)n, c->d_oracles, (int32_t)j,
+                                     (T*)c->d_multi + bucket_off[j], (uint64_t*)(S0 + o_cnt), st)))
                 return rc;
             step_launches += 1;
+            bytes += (double)n;   // each extraction reads the oracle bytes
         }
-        bytes += (double)nb * n;   // each extraction reads the oracle bytes
     }
+    // equality buckets: the value is splitter s_j (row field 4)
+    std::vector<int> tails;
     for (int i = 0; i < m; ++i) {
-        const int64_t j = sr[4 * (size_t)i], kk = sr[4 * (size_t)i + 1], nj = sr[4 * (size_t)i + 2],
-                      eq = sr[4 * (size_t)i + 3];
-        if (!eq) bytes += 2.0 * sizeof(T) * nj;
-        (void)kk;
+        const int64_t* row = sr + MS_ROW * (size_t)i;
+        if (row[3]) {
+            std::memcpy(outb + (size_t)i * sizeof(T), &row[4], sizeof(T));
+        } else {
+            bytes += 2.0 * sizeof(T) * (double)row[2];
+            tails.push_back(i);
+        }
     }
-    // equality buckets: the value is splitter j (1-based), keys -> values
-    for (int i = 0; i < m; ++i) {
-        const int64_t j = sr[4 * (size_t)i], eq = sr[4 * (size_t)i + 3];
-        if (!eq) continue;
-        if ((rc = ss_step_keys_to_values(c, dt, S0 + o_spl + (size_t)(j - 1) * sizeof(K), 1, S0 + o_val, st)))
-            return rc;
-        CK(cudaMemcpyAsync(outb + (size_t)i * sizeof(T), S0 + o_val, sizeof(T), cudaMemcpyDeviceToHost, st));
-        CK(cudaStreamSynchronize(st));   // S0 + o_val is reused by the next equality rank
-        step_launches += 1;
-    }
-    CK(cudaStreamSynchronize(st));
-    // the remaining levels of each rank: single-rank select on its bucket
-    for (int i = 0; i < m; ++i) {
-        const int64_t j = sr[4 * (size_t)i], kk = sr[4 * (size_t)i + 1], nj = sr[4 * (size_t)i + 2],
-                      eq = sr[4 * (size_t)i + 3];
-        if (eq) continue;
-        if ((rc = run_exact<T>(c, (const T*)c->d_multi + bucket_off[j], (u64)nj, (u64)kk,
-                               outb + (size_t)i * sizeof(T), st)))
-            return rc;
-        bytes += c->stats.bytes_algorithmic;
-        launches += c->stats.launches;
+    // the remaining levels of each rank: single-rank selects on its bucket,
+    // MULTI_CH at a time on the child contexts' streams
+    const int nt = (int)tails.size();
+    if (nt) {
+        if ((rc = multi_children(c, nt))) return rc;
+        CK(cudaEventRecord(c->ev_mfork, st));
+        const int nch = std::min(nt, MULTI_CH);
+        for (int w0 = 0; w0 < nt; w0 += nch) {
+            const int wn = std::min(nch, nt - w0);
+            for (int q = 0; q < wn; ++q) {
+                const int i = tails[w0 + q];
+                const int64_t* row = sr + MS_ROW * (size_t)i;
+                ss_context* ch = c->mchild[q];
+                if (w0 == 0) CK(cudaStreamWaitEvent(c->mchild_st[q], c->ev_mfork, 0));
+                if ((rc = run_exact_begin<T>(ch, (const T*)c->d_multi + bucket_off[row[0]], (u64)row[2], (u64)row[1],
+                                             outb + (size_t)i * sizeof(T), c->mchild_st[q])))
+                    return fail(c, rc, ch->err.c_str());
+            }
+            for (int q = 0; q < wn; ++q) {
+                ss_context* ch = c->mchild[q];
+                if ((rc = run_exact_end<T>(ch, c->mchild_st[q]))) return fail(c, rc, ch->err.c_str());
+                bytes += ch->stats.bytes_algorithmic;
+                launches += ch->stats.launches;
+            }
+        }
+        for (int q = 0; q < nch; ++q) {            // later work on the caller's stream follows the tails
+            CK(cudaEventRecord(c->ev_mjoin[q], c->mchild_st[q]));
+            CK(cudaStreamWaitEvent(st, c->ev_mjoin[q], 0));
+        }
     }
     c->launches_total += step_launches;
     std::memset(&c->stats, 0, sizeof(c->stats));
@@ -1307,7 +1522,8 @@ ss_status run_multi(ss_context* c, ss_dtype dt, const T* d, u64 n, int m, const 
     c->stats.n_level[1] = (int64_t)total;
     c->stats.bytes_algorithmic = bytes;
     c->stats.launches = launches + step_launches;
-    c->stats.d2h_bytes = (int64_t)(sizeof(int64_t) * 4 * (size_t)m);
+    c->stats.h2d_bytes = (int64_t)(sizeof(int64_t) * (size_t)m);
+    c->stats.d2h_bytes = (int64_t)(sizeof(int64_t) * MS_ROW * (size_t)m);
     return SS_OK;
 }
 
@@ -1399,7 +1615,7 @@ ss_status run_quick(ss_context* c, const T* d, u64 n, u64 k, void* h_result, int
 
 
 size_t workspace_bytes(const ss_context* c) {
-    size_t b = c->cap_oracles + c->cap_buf[0] + c->cap_buf[1] + c->cap_stage + c->cap_multi + 2 * c->cap_qsbuf +
+    size_t b = c->cap_oracles + c->cap_buf[0] + c->cap_buf[1] + c->cap_win + c->cap_stage + c->cap_multi + 2 * c->cap_qsbuf +
                c->cap_gather[0] + c->cap_gather[1] + c->cap_dist;
     if (c->d_ctl)   // the fixed per-context arrays (ensure_small)
         b += sizeof(LevelCtl) * (SS_MAX_LEVELS + 1) + sizeof(SelectResult) + sizeof(u64) * SS_MAX_LEVELS * MAX_B +

@@ -86,7 +86,7 @@ ss_status run_sharded(ss_context* c, const T* d, u64 n_local, u64 k, void* h_res
     // a level a pass-through or adds one after the hand-off, identically on
     // every rank.
     CK(launch_pdl(init_kernel<T>, dim3(1), dim3(256), 0, st, c->d_ctl, (int)(SS_MAX_LEVELS + 1), c->d_totals,
-                  (int)(SS_MAX_LEVELS * MAX_B), c->d_res, n_local, k, 0, d, 0, (u64)c->cfg.seed, (K*)nullptr));
+                  (int)(SS_MAX_LEVELS * MAX_B), c->d_res, n_local, k, 0, d, 0, (u64)c->cfg.seed, (K*)nullptr, (void*)nullptr));
     CKLAUNCH("init_kernel");
     CK(launch_pdl(dist_sizes_kernel, dim3(1), dim3(32), 0, st, dd + DistLayout::sizes_send, P, R, n_local));
     CKLAUNCH("dist_sizes_kernel");

@@ -35,7 +35,7 @@ def test_header_declares_expected_api():
 def test_library_exports_every_declared_symbol(lib):
     for name in _declared():
         assert hasattr(lib, name), name
-    assert lib.ss_abi_version() == 6
+    assert lib.ss_abi_version() == 7
 
 
 def test_exported_symbols_are_c_linkage(lib):

@@ -1,6 +1,7 @@
-"""The cached CUDA graph of an exact call is keyed on (dtype, n, plan), not on
-the input pointer: the rank k and the input pointer are patched into the
-graph's init node, and level 0's kernels read the input from LevelCtl::src.
+"""The cached CUDA graph of an exact call is keyed on (dtype, plan), not on
+the input pointer or n: the size n, the rank k and the input pointer are
+patched into the graph's init node, and level 0's kernels read the input from
+LevelCtl::src (every kernel reads its level's size from its LevelCtl).
 Calls that rotate over distinct buffers -- including misaligned views, whose
 peeled heads differ -- must each return the oracle's element."""
 import numpy as np
@@ -37,4 +38,25 @@ def test_rotating_buffers_share_one_graph(dtype, fused, cuda_device):
         for i, (x, xd) in enumerate(zip(xs, xds)):
             k = ks[(i + rep) % len(ks)]
             assert _bits(ctx.select(xd, k)) == _bits(oracle.select(x, k)), (i, k, rep)
+    ctx.close()
+
+
+@pytest.mark.parametrize("dtype", [np.float32, np.int64])
+def test_varying_sizes_share_graphs(dtype, cuda_device):
+    """Sizes with the same level plan reuse one graph with n patched; sizes
+    with other plans get their own.  Every call is exact, in any order."""
+    import torch
+    import paper_conf_ipps_ribizela19_b200 as ss
+    ctx = ss.Context(0)
+    kind = "normal" if np.dtype(dtype).kind == "f" else "int"
+    sizes = [(1 << 22) + 3, (1 << 22) + 1001, (1 << 22) - 77777, (1 << 20) + 5, 70000, 5000, (1 << 22) + 5]
+    data = {}
+    for i, n in enumerate(sizes):
+        x = datagen.make(kind, n, dtype, seed=60 + i)
+        data[n] = (x, torch.from_numpy(x).to("cuda:0"))
+    for rep in range(2):
+        for i, n in enumerate(sizes if rep == 0 else sizes[::-1]):
+            x, xd = data[n]
+            for k in (n // 2, datagen.rank(n, i + 3 * rep)):
+                assert _bits(ctx.select(xd, k)) == _bits(oracle.select(x, k)), (n, k, rep)
     ctx.close()
