@@ -1373,6 +1373,46 @@ inline ss_status multi_children(ss_context* c, int want) {
     return SS_OK;
 }
 
+// The per-rank selects of a multi-rank call: exact calls on child contexts,
+// MULTI_CH at a time, each on its own stream after `st`'s work so far; the
+// caller's stream waits for them at the end.
+struct MultiTail {
+    const void* in;
+    u64 n, k;
+    unsigned char* out;   // host result slot
+};
+template <typename T>
+ss_status run_tails(ss_context* c, const std::vector<MultiTail>& tails, cudaStream_t st, double* bytes,
+                    int* launches) {
+    const int nt = (int)tails.size();
+    if (!nt) return SS_OK;
+    ss_status rc;
+    if ((rc = multi_children(c, nt))) return rc;
+    CK(cudaEventRecord(c->ev_mfork, st));
+    const int nch = std::min(nt, MULTI_CH);
+    for (int w0 = 0; w0 < nt; w0 += nch) {
+        const int wn = std::min(nch, nt - w0);
+        for (int q = 0; q < wn; ++q) {
+            const MultiTail& t = tails[w0 + q];
+            ss_context* ch = c->mchild[q];
+            if (w0 == 0) CK(cudaStreamWaitEvent(c->mchild_st[q], c->ev_mfork, 0));
+            if ((rc = run_exact_begin<T>(ch, reinterpret_cast<const T*>(t.in), t.n, t.k, t.out, c->mchild_st[q])))
+                return fail(c, rc, ch->err.c_str());
+        }
+        for (int q = 0; q < wn; ++q) {
+            ss_context* ch = c->mchild[q];
+            if ((rc = run_exact_end<T>(ch, c->mchild_st[q]))) return fail(c, rc, ch->err.c_str());
+            *bytes += ch->stats.bytes_algorithmic;
+            *launches += ch->stats.launches;
+        }
+    }
+    for (int q = 0; q < nch; ++q) {            // later work on the caller's stream follows the tails
+        CK(cudaEventRecord(c->ev_mjoin[q], c->mchild_st[q]));
+        CK(cudaStreamWaitEvent(st, c->ev_mjoin[q], 0));
+    }
+    return SS_OK;
+}
+
 template <typename T>
 ss_status run_multi(ss_context* c, ss_dtype dt, const T* d, u64 n, int m, const int64_t* ks, void* h_res,
                     cudaStream_t st) {
@@ -1485,36 +1525,14 @@ ss_status run_multi(ss_context* c, ss_dtype dt, const T* d, u64 n, int m, const 
             tails.push_back(i);
         }
     }
-    // the remaining levels of each rank: single-rank selects on its bucket,
-    // MULTI_CH at a time on the child contexts' streams
-    const int nt = (int)tails.size();
-    if (nt) {
-        if ((rc = multi_children(c, nt))) return rc;
-        CK(cudaEventRecord(c->ev_mfork, st));
-        const int nch = std::min(nt, MULTI_CH);
-        for (int w0 = 0; w0 < nt; w0 += nch) {
-            const int wn = std::min(nch, nt - w0);
-            for (int q = 0; q < wn; ++q) {
-                const int i = tails[w0 + q];
-                const int64_t* row = sr + MS_ROW * (size_t)i;
-                ss_context* ch = c->mchild[q];
-                if (w0 == 0) CK(cudaStreamWaitEvent(c->mchild_st[q], c->ev_mfork, 0));
-                if ((rc = run_exact_begin<T>(ch, (const T*)c->d_multi + bucket_off[row[0]], (u64)row[2], (u64)row[1],
-                                             outb + (size_t)i * sizeof(T), c->mchild_st[q])))
-                    return fail(c, rc, ch->err.c_str());
-            }
-            for (int q = 0; q < wn; ++q) {
-                ss_context* ch = c->mchild[q];
-                if ((rc = run_exact_end<T>(ch, c->mchild_st[q]))) return fail(c, rc, ch->err.c_str());
-                bytes += ch->stats.bytes_algorithmic;
-                launches += ch->stats.launches;
-            }
-        }
-        for (int q = 0; q < nch; ++q) {            // later work on the caller's stream follows the tails
-            CK(cudaEventRecord(c->ev_mjoin[q], c->mchild_st[q]));
-            CK(cudaStreamWaitEvent(st, c->ev_mjoin[q], 0));
-        }
+    // the remaining levels of each rank: single-rank selects on its bucket
+    std::vector<MultiTail> tl;
+    for (int i : tails) {
+        const int64_t* row = sr + MS_ROW * (size_t)i;
+        tl.push_back({(const T*)c->d_multi + bucket_off[row[0]], (u64)row[2], (u64)row[1],
+                      outb + (size_t)i * sizeof(T)});
     }
+    if ((rc = run_tails<T>(c, tl, st, &bytes, &launches))) return rc;
     c->launches_total += step_launches;
     std::memset(&c->stats, 0, sizeof(c->stats));
     c->stats.levels = 1;

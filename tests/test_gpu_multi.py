@@ -99,3 +99,48 @@ def test_multi_one_pass_and_per_bucket_extraction(ctx, m):
     ks = np.random.default_rng(m).integers(0, n, m).tolist()
     got = ctx.select_multi(torch.from_numpy(x).to("cuda:0"), ks)
     assert np.array_equal(_bits_arr(got), _bits_arr(oracle.select_multi(x, ks)))
+
+
+# ------------------------------------------------ per-rank tails --------
+# The per-rank selects run as exact calls on child contexts (their own
+# streams), with graphs keyed on the plan and n patched per call.
+
+def _check(ctx, x, xd, ks):
+    got = ctx.select_multi(xd, ks)
+    assert np.array_equal(_bits_arr(got), _bits_arr(oracle.select_multi(x, ks))), ks
+    return ctx.stats()
+
+
+@pytest.mark.parametrize("dtype", DTYPES)
+@pytest.mark.parametrize("kind", ["normal", "distinct16", "equal", "specials"])
+def test_multi_few_ranks(ctx, dtype, kind):
+    """4 .. 16 ranks (the bench's regime): shared count, one extraction pass,
+    the per-rank tails concurrently on the child contexts."""
+    import torch
+    n = (1 << 22) + 9
+    x = _gen(kind, n, dtype, seed=71)
+    xd = torch.from_numpy(x).to("cuda:0")
+    rng = np.random.default_rng(72)
+    for ks in ([0, 1, n // 2, n - 1], [n // 3, n // 3 + 1, n // 3 + 2, n // 3 + 50000, 2 * n // 3],
+               rng.integers(0, n, 8).tolist(), rng.integers(0, n, 16).tolist()):
+        _check(ctx, x, xd, ks)
+
+
+def test_multi_sorted_input(ctx):
+    """A sorted input: each extracted bucket comes from one or two CTAs."""
+    import torch
+    n = (1 << 22) + 1
+    x = np.sort(_gen("normal", n, np.float32, seed=74))
+    xd = torch.from_numpy(x).to("cuda:0")
+    _check(ctx, x, xd, [5, n // 4, n // 2, n - 7, 3 * n // 4])
+
+
+def test_multi_rotating_sizes(ctx):
+    """Bucket sizes change from call to call: the per-rank selects reuse their
+    graphs with n patched (graphs keyed on the plan)."""
+    import torch
+    for i, n in enumerate([(1 << 22) + 1, (1 << 22) + 777, (1 << 21) + 5]):
+        x = _gen("normal", n, np.float32, seed=80 + i)
+        xd = torch.from_numpy(x).to("cuda:0")
+        rng = np.random.default_rng(90 + i)
+        _check(ctx, x, xd, rng.integers(0, n, 6).tolist())
