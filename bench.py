@@ -467,6 +467,10 @@ def run_ours(args, rank, world, local_rank):
         kname = "window_kernel (fused count + filter, level 0)"
         k2_bytes = S * n + S * int(last["n_level"][1])
         tkey = f"window_{args.mode}_{args.dtype}_2p{args.log2n}"
+    elif not exact and last.get("spec_levels", 0) & 1:
+        kname = "window_kernel<APX> (approximate: one-pass splitter window, level 0)"
+        k2_bytes = S * n                                   # one read; the window's ranks stay on chip
+        tkey = f"window_approx_{args.dtype}_2p{args.log2n}"
     else:
         kname = "count_kernel (K2, level 0)"
         k2_bytes = (S + (1 if exact else 0)) * n          # read S*n, write n oracle bytes

@@ -99,12 +99,8 @@ struct ss_context {
     // init node (level 0's kernels read the input from LevelCtl::src)
     struct GraphEntry {
         bool used = false;
-        int dt = -1;
-        u64 sig = 0;                          // the plan's signature (levels, fused / directed flags,
-                                              // sample sizes): n itself is patched like k
-        int b0 = 0, bd = 0, s = 0, sd = 0, L = 0, prof = 0;
-        u32 B = 0;
-        u64 seed = 0;
+        u64 key = 0;                          // hash of what the captured chain bakes in (graph_launch):
+                                              // dtype, plan, sample sizes, seed, ...; n itself is patched
         cudaGraph_t graph = nullptr;       // kept: the init node handle belongs to it
         cudaGraphExec_t exec = nullptr;
         cudaGraphNode_t init_node = nullptr;
@@ -114,8 +110,7 @@ struct ss_context {
         size_t k_offset = 0;                  // where k lives in init_store
         size_t n_offset = 0;                  // where n lives in init_store
         size_t d_offset = 0;                  // where the input pointer lives in init_store
-        size_t up_offset = 0;                 // where the top-k output pointer lives (up graphs)
-        bool up = false;                      // top-k graph: level 0 streams the keys above its window
+        size_t up_offset = 0;                 // where the top-k output pointer lives
         int kernels = 0;
         u64 stamp = 0;
     } graphs[8];
@@ -772,6 +767,111 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
     return launch_wsel<T>(c, in, lev, 0, p.B, nullptr, 1, q);
 }
 
+// Launch a call's chain as one cached CUDA graph keyed on `key` (everything
+// the captured kernels bake in: dtype, plan, sample sizes, seed ...): captured
+// on first use (enqueue(capture stream)), then replayed with n, k, the input
+// and the top-k output patched into its init node -- the only kernel that
+// takes them as arguments (the others read LevelCtl).
+template <typename T, typename F>
+ss_status graph_launch(ss_context* c, u64 key, u64 n, u64 k, const T* d, void* up, F&& enqueue, cudaStream_t st) {
+    typedef typename Traits<T>::Key K;
+    ss_context::GraphEntry* ge = nullptr;
+    for (auto& e : c->graphs)
+        if (e.used && e.key == key) ge = &e;
+    if (!ge) {
+        ss_context::GraphEntry* slot = nullptr;           // a free entry, else the least recently used
+        for (auto& e : c->graphs)
+            if (!e.used) { slot = &e; break; }
+        if (!slot) {
+            slot = &c->graphs[0];
+            for (auto& e : c->graphs)
+                if (e.stamp < slot->stamp) slot = &e;
+        }
+        if (slot->exec) cudaGraphExecDestroy(slot->exec);
+        if (slot->graph) cudaGraphDestroy(slot->graph);
+        *slot = ss_context::GraphEntry();
+        const int launches0 = c->launches;
+        CK(cudaStreamBeginCapture(c->cap_st, cudaStreamCaptureModeThreadLocal));
+        const ss_status rc2 = enqueue(c->cap_st);
+        cudaGraph_t g = nullptr;
+        const cudaError_t ec = cudaStreamEndCapture(c->cap_st, &g);
+        if (rc2) {
+            if (g) cudaGraphDestroy(g);
+            return rc2;
+        }
+        CK(ec);
+        cudaGraphExec_t ex = nullptr;
+        const cudaError_t ei = cudaGraphInstantiate(&ex, g, 0);
+        // the init node: the graph's only kernel node running init_kernel<T>
+        size_t nn = 0;
+        cudaGraphGetNodes(g, nullptr, &nn);
+        std::vector<cudaGraphNode_t> nodes(nn);
+        cudaGraphGetNodes(g, nodes.data(), &nn);
+        cudaGraphNode_t init_node = nullptr;
+        cudaKernelNodeParams ip{};
+        for (auto nd : nodes) {
+            cudaGraphNodeType ty;
+            cudaGraphNodeGetType(nd, &ty);
+            if (ty != cudaGraphNodeTypeKernel) continue;
+            cudaKernelNodeParams kp{};
+            if (cudaGraphKernelNodeGetParams(nd, &kp) == cudaSuccess &&
+                kp.func == reinterpret_cast<void*>(init_kernel<T>)) {
+                init_node = nd;
+                ip = kp;
+            }
+        }
+        if (ei != cudaSuccess || !init_node) {
+            cudaGraphDestroy(g);
+            if (ex) cudaGraphExecDestroy(ex);
+            (void)cudaGetLastError();
+            return fail(c, SS_ERR_CUDA, "graph capture of the level chain failed");
+        }
+        slot->used = true;
+        slot->key = key;
+        slot->exec = ex;
+        slot->init_node = init_node;
+        slot->kernels = c->launches - launches0;
+        // private copy of the init arguments (n index 5, k 6, input 8, top-k output 12)
+        slot->init_params = ip;
+        size_t off = 0;
+        const size_t sizes[13] = {sizeof(LevelCtl*), sizeof(int), sizeof(u64*), sizeof(int), sizeof(SelectResult*),
+                                  sizeof(u64), sizeof(u64), sizeof(int), sizeof(const T*), sizeof(int), sizeof(u64),
+                                  sizeof(K*), sizeof(void*)};
+        for (int i = 0; i < 13; ++i) {
+            off = (off + 7) & ~(size_t)7;
+            std::memcpy(slot->init_store + off, ip.kernelParams[i], sizes[i]);
+            slot->init_args[i] = slot->init_store + off;
+            if (i == 5) slot->n_offset = off;
+            if (i == 6) slot->k_offset = off;
+            if (i == 8) slot->d_offset = off;
+            if (i == 12) slot->up_offset = off;
+            off += sizes[i];
+        }
+        slot->init_params.kernelParams = slot->init_args;
+        slot->init_params.extra = nullptr;
+        slot->graph = g;
+        ge = slot;
+        c->launches = launches0;
+    } else {
+        u64 kk = k, nn = n;
+        const T* dd = d;
+        if (std::memcmp(ge->init_store + ge->k_offset, &kk, sizeof(u64)) ||
+            std::memcmp(ge->init_store + ge->n_offset, &nn, sizeof(u64)) ||
+            std::memcmp(ge->init_store + ge->d_offset, &dd, sizeof(const T*)) ||
+            std::memcmp(ge->init_store + ge->up_offset, &up, sizeof(void*))) {   // (unchanged: no update)
+            std::memcpy(ge->init_store + ge->k_offset, &kk, sizeof(u64));
+            std::memcpy(ge->init_store + ge->n_offset, &nn, sizeof(u64));
+            std::memcpy(ge->init_store + ge->d_offset, &dd, sizeof(const T*));
+            std::memcpy(ge->init_store + ge->up_offset, &up, sizeof(void*));
+            CK(cudaGraphExecKernelNodeSetParams(ge->exec, ge->init_node, &ge->init_params));
+        }
+    }
+    ge->stamp = ++c->graph_clock;
+    CK(cudaGraphLaunch(ge->exec, st));
+    c->launches += ge->kernels;
+    return SS_OK;
+}
+
 // top-k tail: the window's keys above the answer, then the copies of it
 template <typename T>
 ss_status enqueue_upper_tail(ss_context* c, bool up, cudaStream_t q) {
@@ -869,125 +969,28 @@ ss_status run_exact_begin(ss_context* c, const T* d, u64 n, u64 k, void* h_resul
     // size from the LevelCtl): graphs are keyed on the plan's signature and
     // n, k, the input and output pointers are patched into the init node.
     const bool graph = c->use_graphs && c->cfg.profile != 1 && c->cfg.profile != 2;
-    ss_context::GraphEntry* ge = nullptr;
-    u64 sig = 1469598103934665603ull;
-    {
-        auto mix = [&](u64 v) { sig = (sig ^ v) * 1099511628211ull; };
+    if (graph) {
+        u64 key = 1469598103934665603ull;
+        auto mix = [&](u64 v) { key = (key ^ v) * 1099511628211ull; };
+        mix(1);                                // exact chain
+        mix((u64)dt_code<T>());
         mix((u64)L);
         mix((u64)s_init);
         mix((u64)pre0);
         for (int l = 0; l < L; ++l) mix((u64)spec_plan[l] | (u64)dir_plan[l] << 1 | (u64)(u32)sf_plan[l] << 2);
-    }
-    if (graph) {
-        for (auto& e : c->graphs)
-            if (e.used && e.dt == dt_code<T>() &&
-                e.sig == sig && e.b0 == b0 && e.bd == bd && e.s == s && e.sd == s_deep && e.L == L &&
-                e.prof == tl_on && e.B == B && e.seed == c->cfg.seed && e.up == up)
-                ge = &e;
-        if (!ge) {
-            ss_context::GraphEntry* slot = nullptr;           // a free entry, else the least recently used
-            for (auto& e : c->graphs)
-                if (!e.used) { slot = &e; break; }
-            if (!slot) {
-                slot = &c->graphs[0];
-                for (auto& e : c->graphs)
-                    if (e.stamp < slot->stamp) slot = &e;
-            }
-            if (slot->exec) cudaGraphExecDestroy(slot->exec);
-            if (slot->graph) cudaGraphDestroy(slot->graph);
-            *slot = ss_context::GraphEntry();
-            const int launches0 = c->launches;
-            CK(cudaStreamBeginCapture(c->cap_st, cudaStreamCaptureModeThreadLocal));
-            ss_status rc2 = enqueue_init(c->cap_st);
-            if (!rc2) rc2 = enqueue_levels(0, c->cap_st);
-            if (!rc2) rc2 = enqueue_upper_tail<T>(c, up, c->cap_st);
-            if (!rc2) rc2 = enqueue_publish(c, c->cap_st);
-            cudaGraph_t g = nullptr;
-            const cudaError_t ec = cudaStreamEndCapture(c->cap_st, &g);
-            if (rc2) {
-                if (g) cudaGraphDestroy(g);
-                return rc2;
-            }
-            CK(ec);
-            cudaGraphExec_t ex = nullptr;
-            const cudaError_t ei = cudaGraphInstantiate(&ex, g, 0);
-            // the init node: the graph's only kernel node running init_kernel<T>
-            size_t nn = 0;
-            cudaGraphGetNodes(g, nullptr, &nn);
-            std::vector<cudaGraphNode_t> nodes(nn);
-            cudaGraphGetNodes(g, nodes.data(), &nn);
-            cudaGraphNode_t init_node = nullptr;
-            cudaKernelNodeParams ip{};
-            for (auto nd : nodes) {
-                cudaGraphNodeType ty;
-                cudaGraphNodeGetType(nd, &ty);
-                if (ty != cudaGraphNodeTypeKernel) continue;
-                cudaKernelNodeParams kp{};
-                if (cudaGraphKernelNodeGetParams(nd, &kp) == cudaSuccess &&
-                    kp.func == reinterpret_cast<void*>(init_kernel<T>)) {
-                    init_node = nd;
-                    ip = kp;
-                }
-            }
-            if (ei != cudaSuccess || !init_node) {
-                cudaGraphDestroy(g);
-                if (ex) cudaGraphExecDestroy(ex);
-                (void)cudaGetLastError();
-                return fail(c, SS_ERR_CUDA, "graph capture of the level chain failed");
-            }
-            slot->used = true;
-            slot->dt = dt_code<T>();
-            slot->sig = sig;
-            slot->b0 = b0; slot->bd = bd; slot->s = s; slot->sd = s_deep; slot->L = L;
-            slot->prof = tl_on; slot->B = B; slot->seed = c->cfg.seed; slot->up = up;
-            slot->exec = ex;
-            slot->init_node = init_node;
-            slot->kernels = c->launches - launches0;
-            // private copy of the init arguments; k is the 7th (index 6)
-            slot->init_params = ip;
-            size_t off = 0;
-            const size_t sizes[13] = {sizeof(LevelCtl*), sizeof(int), sizeof(u64*), sizeof(int), sizeof(SelectResult*),
-                                      sizeof(u64), sizeof(u64), sizeof(int), sizeof(const T*), sizeof(int), sizeof(u64),
-                                      sizeof(K*), sizeof(void*)};
-            for (int i = 0; i < 13; ++i) {
-                off = (off + 7) & ~(size_t)7;
-                std::memcpy(slot->init_store + off, ip.kernelParams[i], sizes[i]);
-                slot->init_args[i] = slot->init_store + off;
-                if (i == 5) slot->n_offset = off;
-                if (i == 6) slot->k_offset = off;
-                if (i == 8) slot->d_offset = off;
-                if (i == 12) slot->up_offset = off;
-                off += sizes[i];
-            }
-            slot->init_params.kernelParams = slot->init_args;
-            slot->init_params.extra = nullptr;
-            slot->graph = g;
-            ge = slot;
-            c->launches = launches0;
-        } else {
-            // the rank and the input pointer are arguments of the init kernel
-            // only (later kernels read level 0's input from LevelCtl::src):
-            // patch them into the cached graph
-            u64 kk = k, nn = n;
-            const T* dd = d;
-            void* uo = up ? (void*)up_out : nullptr;
-            if (std::memcmp(ge->init_store + ge->k_offset, &kk, sizeof(u64)) ||
-                std::memcmp(ge->init_store + ge->n_offset, &nn, sizeof(u64)) ||
-                std::memcmp(ge->init_store + ge->d_offset, &dd, sizeof(const T*)) ||
-                std::memcmp(ge->init_store + ge->up_offset, &uo, sizeof(void*))) {   // (unchanged: no update)
-                std::memcpy(ge->init_store + ge->k_offset, &kk, sizeof(u64));
-                std::memcpy(ge->init_store + ge->n_offset, &nn, sizeof(u64));
-                std::memcpy(ge->init_store + ge->d_offset, &dd, sizeof(const T*));
-                std::memcpy(ge->init_store + ge->up_offset, &uo, sizeof(void*));
-                CK(cudaGraphExecKernelNodeSetParams(ge->exec, ge->init_node, &ge->init_params));
-            }
-        }
-        ge->stamp = ++c->graph_clock;
+        mix((u64)b0); mix((u64)bd); mix((u64)s); mix((u64)s_deep); mix((u64)B);
+        mix((u64)tl_on); mix(c->cfg.seed); mix((u64)up);
+        auto enqueue_all = [&](cudaStream_t q) -> ss_status {
+            ss_status r2 = enqueue_init(q);
+            if (!r2) r2 = enqueue_levels(0, q);
+            if (!r2) r2 = enqueue_upper_tail<T>(c, up, q);
+            if (!r2) r2 = enqueue_publish(c, q);
+            return r2;
+        };
         if (c->host_timing) c->ht[0] += now_us() - t_in;
         const double t_l = c->host_timing ? now_us() : 0.0;
-        CK(cudaGraphLaunch(ge->exec, st));
+        if ((rc = graph_launch<T>(c, key, n, k, d, up ? (void*)up_out : nullptr, enqueue_all, st))) return rc;
         if (c->host_timing) c->ht[1] += now_us() - t_l;
-        c->launches += ge->kernels;
     } else {
         if ((rc = enqueue_init(st))) return rc;
         if ((rc = enqueue_levels(0, st))) return rc;
@@ -1157,31 +1160,36 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     const bool merge = s > WIDE_K1_MAX_S && s % (int)K1C_CHUNK == 0;   // chunk sort + merge rank
     const bool wide = s <= WIDE_K1_MAX_S || merge;
     K* sample0 = s <= WIDE_K1_MAX_S ? reinterpret_cast<K*>(c->d_sample0) : nullptr;
-    CK(launch_pdl(init_kernel<T>, dim3(sample0 ? ((u32)s + 255u) / 256u : 1u), dim3(256), 0, st, c->d_ctl, 2, c->d_totals,
-                  (int)MAX_B, c->d_res, n, k, (int)(c->cfg.profile == 3), d, s, (u64)c->cfg.seed, sample0, (void*)nullptr));
-    CKLAUNCH("init_kernel");
-    ++c->launches;
     // fused one-pass window (approx_window in kernels.cuh) on large inputs;
     // the paper's full count runs only if it cannot decide
     const SpecCfg sp = spec_params(c);
     const bool fw = sp.min_n != ~0ull && n >= sp.min_n;
     K* sorted0 = reinterpret_cast<K*>(c->d_sorted);
-    if (merge) {
-        K* chunks = reinterpret_cast<K*>(c->d_sorted) + MAX_S;   // level 1's slot: scratch here
-        mark(c, 0, 0, 0, st);
-        CK(launch_pdl(sample_chunk_sort_kernel<T>, dim3((u32)s / K1C_CHUNK), dim3(1024), K1C_CHUNK * sizeof(K), st,
-                      d, c->d_ctl, c->d_res, chunks, (u64)c->cfg.seed, 0));
-        CKLAUNCH("sample_chunk_sort_kernel");
-        CK(launch_pdl(sample_merge_rank_kernel<T>, dim3((u32)s / 1024u), dim3(1024), (size_t)s * sizeof(K), st,
-                      c->d_ctl, c->d_res, chunks, s, sorted0, 0));
-        CKLAUNCH("sample_merge_rank_kernel");
-        mark(c, 0, 0, 1, st);
-        c->launches += 2;
-    } else if (wide) {
-        if ((rc = launch_k1_wide<T>(c, d, 0, s, 0, st, sample0))) return rc;
-    } else if ((rc = launch_k1<T>(c, d, 0, s, b, 0, 0, 0, st, fw ? sorted0 : nullptr))) {
-        return rc;
-    }
+    const int tl_on = c->cfg.profile == 3;
+    auto enqueue_head = [&](cudaStream_t q) -> ss_status {   // init, the sorted sample
+        CK(launch_pdl(init_kernel<T>, dim3(sample0 ? ((u32)s + 255u) / 256u : 1u), dim3(256), 0, q, c->d_ctl, 2,
+                      c->d_totals, (int)MAX_B, c->d_res, n, k, tl_on, d, s, (u64)c->cfg.seed, sample0,
+                      (void*)nullptr));
+        CKLAUNCH("init_kernel");
+        ++c->launches;
+        if (merge) {
+            K* chunks = reinterpret_cast<K*>(c->d_sorted) + MAX_S;   // level 1's slot: scratch here
+            mark(c, 0, 0, 0, q);
+            CK(launch_pdl(sample_chunk_sort_kernel<T>, dim3((u32)s / K1C_CHUNK), dim3(1024), K1C_CHUNK * sizeof(K), q,
+                          d, c->d_ctl, c->d_res, chunks, (u64)c->cfg.seed, 0));
+            CKLAUNCH("sample_chunk_sort_kernel");
+            CK(launch_pdl(sample_merge_rank_kernel<T>, dim3((u32)s / 1024u), dim3(1024), (size_t)s * sizeof(K), q,
+                          c->d_ctl, c->d_res, chunks, s, sorted0, 0));
+            CKLAUNCH("sample_merge_rank_kernel");
+            mark(c, 0, 0, 1, q);
+            c->launches += 2;
+        } else if (wide) {
+            if ((rc = launch_k1_wide<T>(c, d, 0, s, 0, q, sample0))) return rc;
+        } else if ((rc = launch_k1<T>(c, d, 0, s, b, 0, 0, 0, q, fw ? sorted0 : nullptr))) {
+            return rc;
+        }
+        return SS_OK;
+    };
     CountArgs a{};
     if (wide) a.image = c->d_image;
     a.ctl = c->d_ctl;
@@ -1197,8 +1205,7 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
     a.lut_stats = c->d_res->lut_stats;
     a.level = 0;
     a.tail = TAIL_APPROX;
-    mark(c, 0, 1, 0, st);
-    if (fw) {
+    auto enqueue_window = [&](cudaStream_t q) -> ss_status {
         CountArgs w = a;
         w.sorted = sorted0;
         w.s = s;
@@ -1206,16 +1213,50 @@ ss_status run_approx(ss_context* c, const T* d, u64 n, u64 k, int b, void* h_res
         w.spec_min_n = sp.min_n;
         w.spec_z = sp.z;
         w.spec_max_frac = 1.0f;
-        if ((rc = launch_window<T, true>(c, H, d, w, st))) return rc;
-        mark(c, 0, 1, 1, st);
+        mark(c, 0, 1, 0, q);
+        if ((rc = launch_window<T, true>(c, H, d, w, q))) return rc;
+        mark(c, 0, 1, 1, q);
         ++c->launches;
+        return SS_OK;
+    };
+    auto enqueue_count = [&](cudaStream_t q) -> ss_status {   // the paper's level-0 count (+ K3/K4 tail)
+        if (!fw) mark(c, 0, 1, 0, q);
+        if (wide && (rc = launch_image<T>(c, H, 0, s, 0, q))) return rc;
+        if ((rc = launch_count<T>(c, H, d, a, q))) return rc;
+        if (!fw) mark(c, 0, 1, 1, q);
+        ++c->launches;
+        return SS_OK;
+    };
+    const bool graph = fw && c->use_graphs && c->cfg.profile != 1 && c->cfg.profile != 2;
+    if (graph) {
+        // the one-pass window decides almost always: one graph (init, sample
+        // sort, window, publish); the count runs after the hand-off only when
+        // the window could not decide (the kernels read n and k from LevelCtl)
+        u64 key = 1469598103934665603ull;
+        auto mix = [&](u64 v) { key = (key ^ v) * 1099511628211ull; };
+        mix(2);                                // approximate chain
+        mix((u64)dt_code<T>()); mix((u64)s); mix((u64)b); mix((u64)tl_on); mix(c->cfg.seed);
+        mix((u64)merge); mix((u64)wide); mix((u64)c->cfg.classify);
+        auto enqueue_all = [&](cudaStream_t q) -> ss_status {
+            ss_status r2 = enqueue_head(q);
+            if (!r2) r2 = enqueue_window(q);
+            if (!r2) r2 = enqueue_publish(c, q);
+            return r2;
+        };
+        if ((rc = graph_launch<T>(c, key, n, k, d, nullptr, enqueue_all, st))) return rc;
+        if ((rc = wait_publish(c, st))) return rc;
+        if (!c->h_res->done) {
+            if ((rc = enqueue_count(st))) return rc;
+            if ((rc = enqueue_publish(c, st))) return rc;
+            if ((rc = wait_publish(c, st))) return rc;
+        }
+    } else {
+        if ((rc = enqueue_head(st))) return rc;
+        if (fw && (rc = enqueue_window(st))) return rc;
+        if ((rc = enqueue_count(st))) return rc;
+        if ((rc = enqueue_publish(c, st))) return rc;
+        if ((rc = wait_publish(c, st))) return rc;
     }
-    if (wide && (rc = launch_image<T>(c, H, 0, s, 0, st))) return rc;
-    if ((rc = launch_count<T>(c, H, d, a, st))) return rc;
-    if (!fw) mark(c, 0, 1, 1, st);
-    ++c->launches;
-    if ((rc = enqueue_publish(c, st))) return rc;
-    if ((rc = wait_publish(c, st))) return rc;
     const SelectResult& r = *c->h_res;
     if (!r.done) return fail(c, SS_ERR_INTERNAL, "approximate select produced no result");
     std::memcpy(h_result, &r.bits, sizeof(T));
