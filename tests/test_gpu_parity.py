@@ -55,6 +55,18 @@ def test_exact_sizes(ctx, dtype, n):
 
 
 @pytest.mark.parametrize("dtype", DTYPES)
+@pytest.mark.parametrize("n", [16385, 40001, 65535, 65536, 65537])
+@pytest.mark.parametrize("kind", ["normal", "distinct16", "specials"])
+def test_small_level_sizes(ctx, dtype, n, kind):
+    """Just above the base case B = 16384 up to the smallest fused level
+    (spec_min_n = 2^16): one paper or fused level, then the cluster base case."""
+    x = _gen(kind, n, dtype, seed=n + 3)
+    xd = _dev(x)
+    for k in _ranks(n, n + 1) + [n // 3, n - 2]:
+        assert _bits(ctx.select(xd, k)) == _bits(oracle.select(x, k)), (n, k, kind)
+
+
+@pytest.mark.parametrize("dtype", DTYPES)
 @pytest.mark.parametrize("kind", ["uniform", "normal", "exponential", "distinct16", "distinct128",
                                   "distinct1024", "equal", "perm", "specials"])
 def test_exact_distributions(ctx, dtype, kind):
