@@ -271,9 +271,12 @@ def _workload_label(args, b, world, levels):
                 f"(2 splitters from a 4096-key sample) per rank, then gather + single-GPU b={b} levels")
     if args.fused == 0:
         return f"k=N/2, the paper's level on every level: b={b} tree, oracle bytes, filter kernel"
-    return (f"k=N/2; levels with n_l >= 2^22 run the fused window (2 splitters from the sorted sample, "
-            f"count + filter in one pass), smaller levels the paper's b={b} tree + oracle-byte filter; "
-            f"level sizes {levels}")
+    return (f"k=N/2; level 0: fused window [klo, khi) from a 16384-key sample (two order statistics by "
+            f"digit narrowing, K1w) -- one pass counts #{{x < klo}} and copies the window (reading R21); "
+            f"deeper fused levels directed by the previous level's 1024-bin key histogram (reading R28); "
+            f"levels below 2^16 elements the paper's b={b} tree + oracle-byte filter; base case on an "
+            f"8-CTA cluster; level sizes {levels} (a trailing 0: the answer came from a one-key bin, "
+            f"an equality exit)")
 
 
 def run_ours(args, rank, world, local_rank):

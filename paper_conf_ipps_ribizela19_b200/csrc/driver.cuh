@@ -46,6 +46,7 @@ struct ExactPlan {
     const void* sample0;              // sample keys of level lev_first gathered ahead (or NULL)
     int lev_first;
     void* out0;                       // top-k call: level 0 writes its window here (d_win), else NULL
+    u32 kw_grid[SS_MAX_LEVELS];       // fused level l's window_kernel grid (0: one CTA per SM)
 };
 
 // ss_select_multi: per-rank tails run as exact calls on child contexts, each
@@ -170,6 +171,7 @@ struct ss_context {
     size_t cap_win = 0;
     bool up_used = false;            // the last run_exact ran the one-pass top-k path
     ExactCall call{};                // the exact call in flight (run_exact_begin .. run_exact_end)
+    bool shared_gpu = false;         // a child context of ss_select_multi: small levels on part of the GPU
     bool host_timing = false;
     double ht[5] = {};
     long long ht_n = 0;
@@ -335,7 +337,7 @@ ss_status launch_count(ss_context* c, int H, const T* in, CountArgs& a, cudaStre
 // fused count + filter kernel: one CTA per SM, KW_SMEM bytes (TMA ring + stash)
 template <typename T, bool APX = false, bool UP = false>
 ss_status launch_window(ss_context* c, int /*H*/, const T* in, CountArgs a, cudaStream_t st) {
-    a.grid = (u32)c->sms * (u32)KW_MINB;
+    if (!a.grid) a.grid = (u32)c->sms * (u32)KW_MINB;   // (a small planned level may take fewer CTAs)
     bool& attr_set = c->kw_attr[dt_code<T>() - 1][APX ? 1 : UP ? 2 : 0];
     if (!attr_set) {
         CK(cudaFuncSetAttribute(window_kernel<T, APX, UP>, cudaFuncAttributeMaxDynamicSharedMemorySize,
@@ -528,7 +530,7 @@ inline double window_frac(float z, int s) {
 // caught on the device (the final level flags "incomplete") and more levels
 // are enqueued.
 int expected_levels(const ss_context* c, u64 n, int b0, int bd, u32 B, bool* spec_plan, int* sf_plan,
-                    bool* dir_plan) {
+                    bool* dir_plan, double* est = nullptr) {
     const SpecCfg sp = spec_params(c);
     const double pad = (double)c->sms * 32.0;
     int L = 0;
@@ -549,6 +551,7 @@ int expected_levels(const ss_context* c, u64 n, int b0, int bd, u32 B, bool* spe
         if (spec_plan) spec_plan[L] = spec;
         if (sf_plan) sf_plan[L] = sf;
         if (dir_plan) dir_plan[L] = dir;
+        if (est) est[L] = m;
         m = dir ? m * 4.0 / KW_HB + pad : spec ? m * 1.2 * f + pad : m * 1.5 / b;
         prev_fused = spec;
         ++L;
@@ -629,6 +632,8 @@ ss_status launch_image(ss_context* c, int H, int lev, int s, int fixup, cudaStre
 // level l > p.lev_first reads the buffer level l-1 wrote (d_buf[(l-1) & 1]).
 
 
+constexpr double KW_CTA_ELEMS = 32768.0;     // elements per window CTA on a small planned level
+
 // The buffer level `lev` writes (and level lev + 1 reads).
 inline void* level_out(const ss_context* c, const ExactPlan& p, int lev) {
     return lev == 0 && p.out0 ? p.out0 : c->d_buf[lev & 1];
@@ -696,6 +701,7 @@ ss_status enqueue_exact_levels(ss_context* c, const ExactPlan& p, const T* first
             w.hist = lev + 1 < p.L && p.dir_plan[lev + 1];
             w.dir_level = p.dir_plan[lev];
             w.totals = c->d_totals + (size_t)lev * MAX_B;   // the hist bins (zeroed by init)
+            w.grid = p.kw_grid[lev];
             mark(c, lev, 1, 0, q);
             if (lev == 0 && p.out0) {          // top-k: also stream the keys above the window out
                 if ((rc = launch_window<T, false, true>(c, H, in, w, q))) return rc;
@@ -911,7 +917,8 @@ ss_status run_exact_begin(ss_context* c, const T* d, u64 n, u64 k, void* h_resul
     bool spec_plan[SS_MAX_LEVELS] = {};
     int sf_plan[SS_MAX_LEVELS] = {};
     bool dir_plan[SS_MAX_LEVELS] = {};
-    int L = expected_levels(c, n, b0, bd, B, spec_plan, sf_plan, dir_plan);
+    double est[SS_MAX_LEVELS] = {};
+    int L = expected_levels(c, n, b0, bd, B, spec_plan, sf_plan, dir_plan, est);
     const int sf = sf_plan[0] ? sf_plan[0] : fused_sample(c->cfg, 0);
     // top-k (§IV.I): a fused level 0 also streams the keys above its window to
     // up_out and keeps its window in d_win for the tail kernels
@@ -959,6 +966,16 @@ ss_status run_exact_begin(ss_context* c, const T* d, u64 n, u64 k, void* h_resul
     plan.sample0 = sample0;
     plan.lev_first = 0;
     plan.out0 = up ? c->d_win : nullptr;
+    // on a child context of ss_select_multi (several selects in flight
+    // together) a small fused level runs on a quarter of the SMs or more,
+    // ~KW_CTA_ELEMS elements per CTA, so the per-rank tails share the GPU
+    // instead of queueing behind each other's full-GPU grids (measured: m = 8
+    // 0.72 -> 0.68 ms; a lone small select is faster on the full grid)
+    for (int l = 0; l < L && c->shared_gpu; ++l) {
+        const u32 full = (u32)c->sms * (u32)KW_MINB, quarter = std::max<u32>(1, full / 4);
+        const double want = std::ceil(est[l] / KW_CTA_ELEMS);
+        plan.kw_grid[l] = want >= (double)full ? 0u : std::max<u32>(quarter, (u32)want);
+    }
     auto enqueue_levels = [&](int lev0, cudaStream_t q) -> ss_status {
         plan.L = L;
         return enqueue_exact_levels<T>(c, plan, d, lev0, q);
@@ -977,7 +994,8 @@ ss_status run_exact_begin(ss_context* c, const T* d, u64 n, u64 k, void* h_resul
         mix((u64)L);
         mix((u64)s_init);
         mix((u64)pre0);
-        for (int l = 0; l < L; ++l) mix((u64)spec_plan[l] | (u64)dir_plan[l] << 1 | (u64)(u32)sf_plan[l] << 2);
+        for (int l = 0; l < L; ++l)
+            mix((u64)spec_plan[l] | (u64)dir_plan[l] << 1 | (u64)(u32)sf_plan[l] << 2 | (u64)plan.kw_grid[l] << 20);
         mix((u64)b0); mix((u64)bd); mix((u64)s); mix((u64)s_deep); mix((u64)B);
         mix((u64)tl_on); mix(c->cfg.seed); mix((u64)up);
         auto enqueue_all = [&](cudaStream_t q) -> ss_status {
@@ -1403,6 +1421,7 @@ inline ss_status multi_children(ss_context* c, int want) {
         if (!c->mchild[i]) {
             ss_status rc = ss_create(c->device, &c->mchild[i]);
             if (rc) return fail(c, rc, "select_multi: child context");
+            c->mchild[i]->shared_gpu = true;
             CK(cudaStreamCreateWithFlags(&c->mchild_st[i], cudaStreamNonBlocking));
             CK(cudaEventCreateWithFlags(&c->ev_mjoin[i], cudaEventDisableTiming));
         }
