@@ -144,6 +144,17 @@ struct TimelineScope {
     }
 };
 
+// Phase stamp of a kernel (profile = 3 diagnostics): slot [0] = ~earliest,
+// [1] = latest %globaltimer over the CTAs that pass it (slots 90.. are free:
+// levels 30 and 31 never run).
+__device__ __forceinline__ void tl_phase(SelectResult* r, int slot) {
+    if (r && r->tl_on && threadIdx.x == 0) {
+        const u64 t = gtimer();
+        atomicMax(reinterpret_cast<unsigned long long*>(r->tl[slot]), ~t);
+        atomicMax(reinterpret_cast<unsigned long long*>(r->tl[slot] + 1), t);
+    }
+}
+
 // ------------------------------------------------------------ chunking ----
 // Element -> CTA mapping shared by the count (K2) and filter (K5) kernels;
 // the filter must see exactly the count's partition so that the K3 offsets

@@ -3,7 +3,9 @@
 # NEXT rows + rotating buffers), the ncu launch list of the bench command,
 # full captures of the top kernels, compute-sanitizer runs.  Output under
 # gpurun_out/ev_*; copy what is judged to profiles/.
-#   usage: bash scripts/gpu_round_evidence.sh [part...]   (parts: smoke tests bench configs ncu sanitize)
+#   usage: bash scripts/gpu_round_evidence.sh [part...]
+#   parts: smoke tests bench configs ncu sanitize (default) and next small (NEXT-1/NEXT-2 sweeps,
+#   small-n device timelines)
 cd "${GRAFT_REPO_ROOT:-.}"
 mkdir -p gpurun_out
 parts="${*:-smoke tests bench configs ncu sanitize}"
@@ -38,6 +40,22 @@ if has ncu; then
   SS_CFG='{"fused_filter": 0}' timeout 900 ncu --set full --clock-control none --import-source on \
     -k regex:"count_kernel|filter_kernel" -s 0 -c 2 -o gpurun_out/ev_full_paper python scripts/profile_one.py 28 \
     > gpurun_out/ev_ncu_full_paper.log 2>&1
+fi
+if has next; then
+  # NEXT-1 top-k on both paths at several output sizes; NEXT-2 at several m; its launch list
+  for uc in 1048576 16777216 67108864 134217728; do
+    timeout 300 python bench.py --no-cpu --mode upper --upper-count $uc > gpurun_out/ev_next_up1_$uc.log 2>&1
+    timeout 300 python bench.py --no-cpu --mode upper --upper-count $uc --cfg '{"upper_onepass": 0}' \
+      > gpurun_out/ev_next_up0_$uc.log 2>&1
+  done
+  for r in 4 8 16 64; do timeout 300 python bench.py --no-cpu --mode multi --ranks $r > gpurun_out/ev_next_multi$r.log 2>&1; done
+  timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/ev_next_multi8_launches.csv \
+    python bench.py --no-cpu --mode multi --ranks 8 --steps 2 --warmup 3 --e2e-steps 1 > /dev/null 2>&1
+fi
+if has small; then
+  # device timelines (profile = 3 stamps) of small selections and of the approximate variant
+  for L in 16 20 24 28; do TL_DEBUG=1 timeout 120 python scripts/timeline.py $L 256; done > gpurun_out/ev_small_tl.log 2>&1
+  for b in 256 1024; do timeout 120 python scripts/timeline.py 28 $b approx; done >> gpurun_out/ev_small_tl.log 2>&1
 fi
 if has sanitize; then
   nvcc -O2 -std=c++17 -gencode arch=compute_100a,code=sm_100a -I include -o build/sanitize_driver scripts/sanitize_driver.cu \

@@ -26,7 +26,7 @@ acc = None
 for _ in range(R):
     run()
     st = ctx.stats()
-    tl = np.array(ctx.raw_tl(), dtype=np.float64)[:8]
+    tl = np.array(ctx.raw_tl(), dtype=np.float64)
     acc = tl if acc is None else acc + tl
 tl = acc / R
 names = ["K1", "K2", "K5"]
@@ -34,12 +34,12 @@ if os.environ.get("WS_DEBUG"):
     import ctypes
     raw = np.array(ctx.raw_tl(), dtype=np.float64)   # us after init, last call only
     print("  K1w phases (us after init, last call):", [round(raw[(80 + i) // 3][(80 + i) % 3][1], 2) for i in range(6)])
-if os.environ.get("TL_DEBUG"):
-    for sl, nm in ((93, "L1K2 cta start"), (90, "L1K2 prologue end"), (91, "L1K2 main end"), (92, "L1K2 ticket")):
+if os.environ.get("TL_DEBUG"):       # window_kernel phase stamps of level 1 (tl_phase)
+    for sl, nm in ((90, "L1 window: setup done"), (91, "L1 window: stream done"), (92, "L1 window: ticket")):
         l, q = divmod(sl, 3)
         print(f"  {nm}: first {tl[l][q][0]:8.1f}  last {tl[l][q][1]:8.1f}")
 print(f"n=2^{log2n} b={b} b_deep={bd} {mode}: n_level={st['n_level']}  (mean of {R} calls, us after init)")
-for l in range(tl.shape[0]):
+for l in range(min(8, tl.shape[0])):
     for q in range(3):
         s0, s1 = tl[l][q]
         if s0 >= 0 and s1 > 0:
