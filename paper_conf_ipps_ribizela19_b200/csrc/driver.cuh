@@ -504,14 +504,17 @@ SpecCfg spec_params(const ss_context* c) {
 }
 
 // Fused-level sample sizes (K1w): the configured sample_size if set (at least
-// 1024), else 16384 at level 0 -- the window is ~6 z / sqrt(s) of the level,
-// and level 0's window decides the largest write and the next level's size --
-// and, deeper, the smallest of 4096 / 8192 / 16384 whose expected window fits
-// the base case (saving a whole level), else 4096: K1w runs on one CTA and
-// its cost grows with s.
-inline int fused_sample(const ss_config& cfg, int level) {
+// 1024), else at level 0 16384 for large inputs -- the window is ~6 z /
+// sqrt(s) of the level, and level 0's window decides the largest write and
+// the next level's size -- and 4096 up to 2^25 elements, where K1w's cost
+// (12.5 vs 7.8 us on B200) outweighs the larger window (measured device time
+// 2^16: 30 -> 26 us, 2^20: 40.6 -> 37.6 us, 2^24: 51 -> 47 us); deeper, the
+// smallest of 4096 / 8192 / 16384 whose expected window fits the base case
+// (saving a whole level), else 4096.
+constexpr u64 SMALL_L0_SAMPLE_MAX_N = (u64)1 << 25;
+inline int fused_sample(const ss_config& cfg, int level, u64 n) {
     if (cfg.sample_size > 0) return std::max(1024, std::min(cfg.sample_size, 16384));
-    return level ? 4096 : 16384;
+    return level || n <= SMALL_L0_SAMPLE_MAX_N ? 4096 : 16384;
 }
 
 inline double window_frac(float z, int s) {
@@ -538,7 +541,7 @@ int expected_levels(const ss_context* c, u64 n, int b0, int bd, u32 B, bool* spe
     bool prev_fused = false;
     while (m > (double)B && L < SS_MAX_LEVELS - 2) {
         const int b = L ? bd : b0;
-        int sf = fused_sample(c->cfg, L);
+        int sf = fused_sample(c->cfg, L, n);
         if (L && c->cfg.sample_size <= 0)
             for (int cand = 4096; cand <= 16384; cand *= 2)
                 if (m * 1.1 * window_frac(sp.z, cand) + pad / 2 <= (double)B) {
@@ -919,7 +922,7 @@ ss_status run_exact_begin(ss_context* c, const T* d, u64 n, u64 k, void* h_resul
     bool dir_plan[SS_MAX_LEVELS] = {};
     double est[SS_MAX_LEVELS] = {};
     int L = expected_levels(c, n, b0, bd, B, spec_plan, sf_plan, dir_plan, est);
-    const int sf = sf_plan[0] ? sf_plan[0] : fused_sample(c->cfg, 0);
+    const int sf = sf_plan[0] ? sf_plan[0] : fused_sample(c->cfg, 0, n);
     // top-k (§IV.I): a fused level 0 also streams the keys above its window to
     // up_out and keeps its window in d_win for the tail kernels
     const bool up = up_out && L > 0 && spec_plan[0];
