@@ -144,11 +144,15 @@ struct TimelineScope {
     }
 };
 
-// Phase stamp of a kernel (profile = 3 diagnostics): slot [0] = ~earliest,
-// [1] = latest %globaltimer over the CTAs that pass it (slots 90.. are free:
-// levels 30 and 31 never run).
+// Phase stamp of a kernel (profile = 3 diagnostics, compiled in only with
+// -DSS_PHASE_STAMPS=1: a stamp costs the stamping warp a global round trip):
+// slot [0] = ~earliest, [1] = latest %globaltimer over the CTAs that pass it
+// (slots 80.. are free: levels >= 27 never run).
+#ifndef SS_PHASE_STAMPS
+#define SS_PHASE_STAMPS 0
+#endif
 __device__ __forceinline__ void tl_phase(SelectResult* r, int slot) {
-    if (r && r->tl_on && threadIdx.x == 0) {
+    if (SS_PHASE_STAMPS && r && r->tl_on && threadIdx.x == 0) {
         const u64 t = gtimer();
         atomicMax(reinterpret_cast<unsigned long long*>(r->tl[slot]), ~t);
         atomicMax(reinterpret_cast<unsigned long long*>(r->tl[slot] + 1), t);

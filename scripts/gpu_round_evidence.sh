@@ -54,7 +54,12 @@ if has next; then
 fi
 if has small; then
   # device timelines (profile = 3 stamps) of small selections and of the approximate variant
-  for L in 16 20 24 28; do TL_DEBUG=1 timeout 120 python scripts/timeline.py $L 256; done > gpurun_out/ev_small_tl.log 2>&1
+  for L in 16 20 24 28; do timeout 120 python scripts/timeline.py $L 256; done > gpurun_out/ev_small_tl.log 2>&1
+  # phase stamps (K1w of level 0, the level-1 window) from a stamped build of the library
+  SS_NVCC_EXTRA=-DSS_PHASE_STAMPS=1 python -c "from paper_conf_ipps_ribizela19_b200 import build as b; b.build(out='build/lib_stamps.so')" \
+    > gpurun_out/ev_small_stamps_build.log 2>&1
+  for L in 24 28; do SS_LIB=build/lib_stamps.so WS_DEBUG=1 TL_DEBUG=1 timeout 120 python scripts/timeline.py $L 256; done \
+    >> gpurun_out/ev_small_tl.log 2>&1
   for b in 256 1024; do timeout 120 python scripts/timeline.py 28 $b approx; done >> gpurun_out/ev_small_tl.log 2>&1
 fi
 if has sanitize; then

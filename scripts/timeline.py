@@ -1,5 +1,8 @@
 """Device timeline of one selection (profile=3: %globaltimer stamps inside the
-kernels, PDL overlap intact).  `python scripts/timeline.py [log2n] [b] [mode]`"""
+kernels, PDL overlap intact).  `python scripts/timeline.py [log2n] [b] [mode]`
+WS_DEBUG=1 / TL_DEBUG=1 print the phase stamps of level 0's K1w / level 1's
+window kernel; they need a library built with SS_NVCC_EXTRA=-DSS_PHASE_STAMPS=1
+(e.g. into build_variants/ and loaded with SS_LIB=...)."""
 import os, sys, time
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import numpy as np, torch
@@ -30,10 +33,12 @@ for _ in range(R):
     acc = tl if acc is None else acc + tl
 tl = acc / R
 names = ["K1", "K2", "K5"]
-if os.environ.get("WS_DEBUG"):
-    import ctypes
-    raw = np.array(ctx.raw_tl(), dtype=np.float64)   # us after init, last call only
-    print("  K1w phases (us after init, last call):", [round(raw[(80 + i) // 3][(80 + i) % 3][1], 2) for i in range(6)])
+if os.environ.get("WS_DEBUG"):        # level-0 K1w phase stamps (tl_phase, last CTA to pass)
+    names_k1w = ["keys loaded", "min/max", "pass 1", "pass 2", "pass 3", "candidates", "ranked"]
+    for i, nm in enumerate(names_k1w):
+        l, q = divmod(80 + i, 3)
+        if tl[l][q][1] > 0:
+            print(f"  K1w {nm}: first {tl[l][q][0]:8.1f}  last {tl[l][q][1]:8.1f}")
 if os.environ.get("TL_DEBUG"):       # window_kernel phase stamps of level 1 (tl_phase)
     for sl, nm in ((90, "L1 window: setup done"), (91, "L1 window: stream done"), (92, "L1 window: ticket")):
         l, q = divmod(sl, 3)
