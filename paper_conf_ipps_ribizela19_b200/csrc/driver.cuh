@@ -1444,6 +1444,21 @@ struct MultiTail {
     u64 n, k;
     unsigned char* out;   // host result slot
 };
+// After a failed tail the children may hold launched calls nobody waits for
+// (their publish counters would run ahead of the host's): drop them all; the
+// next multi-rank call creates fresh ones.
+inline void multi_children_reset(ss_context* c) {
+    for (int i = 0; i < MULTI_CH; ++i) {
+        if (c->mchild_st[i]) cudaStreamSynchronize(c->mchild_st[i]);
+        if (c->mchild[i]) ss_destroy(c->mchild[i]);
+        if (c->mchild_st[i]) cudaStreamDestroy(c->mchild_st[i]);
+        if (c->ev_mjoin[i]) cudaEventDestroy(c->ev_mjoin[i]);
+        c->mchild[i] = nullptr;
+        c->mchild_st[i] = nullptr;
+        c->ev_mjoin[i] = nullptr;
+    }
+}
+
 template <typename T>
 ss_status run_tails(ss_context* c, const std::vector<MultiTail>& tails, cudaStream_t st, double* bytes,
                     int* launches) {
@@ -1451,6 +1466,11 @@ ss_status run_tails(ss_context* c, const std::vector<MultiTail>& tails, cudaStre
     if (!nt) return SS_OK;
     ss_status rc;
     if ((rc = multi_children(c, nt))) return rc;
+    auto failed = [&](ss_context* ch, ss_status r) -> ss_status {
+        const std::string msg = ch->err;
+        multi_children_reset(c);
+        return fail(c, r, msg.c_str());
+    };
     CK(cudaEventRecord(c->ev_mfork, st));
     const int nch = std::min(nt, MULTI_CH);
     for (int w0 = 0; w0 < nt; w0 += nch) {
@@ -1460,11 +1480,11 @@ ss_status run_tails(ss_context* c, const std::vector<MultiTail>& tails, cudaStre
             ss_context* ch = c->mchild[q];
             if (w0 == 0) CK(cudaStreamWaitEvent(c->mchild_st[q], c->ev_mfork, 0));
             if ((rc = run_exact_begin<T>(ch, reinterpret_cast<const T*>(t.in), t.n, t.k, t.out, c->mchild_st[q])))
-                return fail(c, rc, ch->err.c_str());
+                return failed(ch, rc);
         }
         for (int q = 0; q < wn; ++q) {
             ss_context* ch = c->mchild[q];
-            if ((rc = run_exact_end<T>(ch, c->mchild_st[q]))) return fail(c, rc, ch->err.c_str());
+            if ((rc = run_exact_end<T>(ch, c->mchild_st[q]))) return failed(ch, rc);
             *bytes += ch->stats.bytes_algorithmic;
             *launches += ch->stats.launches;
         }
