@@ -68,6 +68,9 @@ struct ExactCall {
     ExactPlan plan;
 };
 
+#ifndef SS_USE_GRAPHS
+#define SS_USE_GRAPHS 1
+#endif
 struct ss_context {
     int device = 0;
     int sms = 0;
@@ -117,7 +120,7 @@ struct ss_context {
     } graphs[8];
     u64 graph_clock = 0;
     cudaStream_t cap_st = nullptr;   // capture stream (graphs are captured off the caller's stream)
-    bool use_graphs = true;
+    bool use_graphs = SS_USE_GRAPHS != 0;   // (-DSS_USE_GRAPHS=0: every call launches its kernels directly)
     // record of the last ss_step_count (per-CTA counts feed ss_step_filter)
     const void* step_ptr = nullptr;
     u64 step_n = 0;
