@@ -93,6 +93,9 @@ struct LevelCtl {
     void* up_out;   // level 0 of a top-k call (§IV.I): the caller's output of the n - k largest
                     // elements (written by the init kernel, patched like src); NULL otherwise
     u64 ucnt;       // top-k: elements written to up_out so far (the keys above the answer)
+    u64 hlo, hspan; // fused level whose window runs to the top / bottom of the key range: its
+                    // histogram bins [hlo, hlo + hspan) (the sample's keys), the first bin also
+                    // taking the window's keys below hlo, the last those above; hspan 0 = the window
 };
 
 struct SelectResult {
